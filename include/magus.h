@@ -1,0 +1,270 @@
+/*
+ * magus.h -- C-ABI of libmagus: a B200 (sm_100a) batch replay of the MAGUS
+ * uncore-frequency decision loop (Zheng, Sultanov, Papka, Lan, "Minimizing
+ * Power Waste in Heterogenous Computing via Adaptive Uncore Scaling", SC'25).
+ *
+ * Citations are P@<byte offset> into the paper text (PAPER.md is one line, so
+ * a byte offset is the only precise locator), plus the section / algorithm.
+ *
+ *   Alg. 1  Memory Throughput Trend Prediction ........ P@20631 (Sec. 3.1)
+ *   Alg. 2  High Frequency Detection ................... P@21063 (Sec. 3.2)
+ *   Alg. 3  MDFS (combination + step rule) ............. P@25445 (Sec. 3.3)
+ *   init: uncore at max, 10-cycle fill, tune list = 10 zeros
+ *                                              P@23755, P@23939, P@24182
+ *   default thresholds 200 / 500 / 0.4, 0.2 s ........... P@25197 (Sec. 3.3)
+ *   Pareto default 300 / 500 / 0.4 ...................... P@44170 (Sec. 6.4)
+ *
+ * Readings of the paper that the library implements (all listed with their
+ * reasons in DESIGN.md section 3): dec_threshold is signed (-500); the first
+ * MDFS round is t = W; Alg. 3's garbled lines 12-14 are "else status <- 0";
+ * a decision made after sample t governs interval t+1; open loop.
+ *
+ * The energy / slowdown accounting ("model M") is an
+ * ASSUMPTION: the paper measures energy with RAPL/NVML (P@31772) and does not
+ * model it.
+ *
+ * Conventions for every call:
+ *   - Returns magus_status; MAGUS_OK == 0.
+ *   - All arguments are validated before anything is launched.  On error no
+ *     output is written and magus_last_error(ctx) holds a one-line reason.
+ *   - Device pointers are raw CUDA device addresses owned by the caller (the
+ *     Python binding allocates them through torch).  The library never frees
+ *     caller memory.  The context owns its scratch memory (grown on demand,
+ *     freed by magus_destroy).
+ *   - The CUDA stream given to magus_init (or magus_set_stream) is borrowed;
+ *     device work is enqueued on it asynchronously.  Calls that return host
+ *     values synchronise that stream and say so.
+ *   - One context per host thread.
+ */
+#ifndef MAGUS_H_
+#define MAGUS_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MAGUS_ABI_VERSION 1
+
+typedef struct magus_ctx_s* magus_ctx;
+
+typedef enum {
+  MAGUS_OK = 0,
+  MAGUS_ERR_INVALID_ARG = 1,
+  MAGUS_ERR_NOT_INITIALIZED = 2,
+  MAGUS_ERR_CUDA = 3,
+  MAGUS_ERR_NCCL = 4,
+  MAGUS_ERR_OOM = 5,
+  MAGUS_ERR_UNSUPPORTED = 6,
+  MAGUS_ERR_NO_FEASIBLE = 7
+} magus_status;
+
+/* One policy configuration = the parameters of Alg. 1-3.
+ * Validation: window >= 2; 1 <= history <= 64; deriv_len finite and > 0;
+ * tau_inc, tau_dec finite; t_hi > 0 and not NaN (t_hi > 1 disables Alg. 2). */
+typedef struct {
+  int32_t window;    /* W = |mem_throughput_ls|. Paper: not stated; reading 10
+                        (filled during the 10-cycle init, P@23939-P@24050).   */
+  int32_t history;   /* H = |uncore_tune_ls|. Paper: 10 zeros (P@24182).     */
+  double  deriv_len; /* L = direv_length, the divisor of Alg. 1 line 3.
+                        Paper: not stated; reading L = W (P@20695).          */
+  double  tau_inc;   /* Alg. 1: d >  tau_inc -> +1. Paper 200 (P@25197).     */
+  double  tau_dec;   /* Alg. 1: d <  tau_dec -> -1. SIGNED: paper "500" is
+                        read as -500 (reading R1).                 */
+  double  t_hi;      /* Alg. 2: s/H >= t_hi -> high-frequency. Paper 0.4.    */
+} magus_policy;
+
+/* Platform + accounting model M (an assumption).
+ * Validation: 1 <= ratio_min < ratio_max <= 127; dt_s > 0; bw_max_mbs > 0;
+ * beta >= 0; all doubles finite; powers/energies >= 0. */
+typedef struct {
+  int32_t ratio_min;      /* uncore ratio, 100 MHz units: 8 (0.8 GHz)        */
+  int32_t ratio_max;      /* 22 (2.2 GHz) Intel+A100, P@29320; 25 Max1550    */
+  double  dt_s;           /* sampling interval, 0.2 s (P@44789)              */
+  double  bw_max_mbs;     /* memory-path capacity at ratio_max (MB/s);
+                             capacity at ratio l is bw_max * l / ratio_max   */
+  double  beta;           /* memory-boundness of the stretch                 */
+  double  p_other_w;      /* power not attributable to the uncore (W)       */
+  double  p_unc_min_w;    /* uncore power at ratio_min (W)                   */
+  double  p_unc_max_w;    /* uncore power at ratio_max (W); 82 W range from
+                             Fig. 2 (P@12253)                                */
+  double  e_switch_j;     /* energy per frequency change ("negligible", 0)   */
+  double  t_switch_s;     /* time per frequency change (0)                   */
+  double  slowdown_bound; /* 0.05, the "<5 % performance loss" (P@1715)      */
+} magus_platform;
+
+/* Result per (config, trace).  Integer counters are exact; time/energy are
+ * model M evaluated from them in a fixed fp64 operation order.  104 bytes. */
+typedef struct {
+  int64_t  n_events;      /* rounds with trend != 0 (Alg. 3 l.17/22 push 1)  */
+  int64_t  n_hi_rounds;   /* rounds with high_freq_status = 1 (l.10)         */
+  int64_t  n_msr_writes;  /* tune_uncore_freq calls (l.11, l.19, l.25)       */
+  int64_t  n_changes;     /* t in [1,T): dec[t] != dec[t-1]                  */
+  int64_t  n_min_dec;     /* #t with dec[t] = ratio_min                      */
+  int64_t  n_min_int;     /* #t whose interval ran at ratio_min (l_t = dec[t-1]) */
+  uint64_t q_min;         /* sum of quantised stretch over intervals at min  */
+  uint64_t q_max;         /* same over intervals at max                      */
+  uint64_t digest;        /* sum_w word_w * (mix64(w)|1) mod 2^64 over the
+                             32-step decision words          */
+  double   time_s;        /* modelled runtime under MAGUS                    */
+  double   energy_j;      /* modelled energy under MAGUS                     */
+  double   slowdown;      /* time_s / base.time_s - 1 (>= 0 exactly)         */
+  int32_t  viol;          /* slowdown > slowdown_bound                       */
+  int32_t  reserved;
+} magus_summary;
+
+/* Config-independent baseline per trace: uncore pinned at ratio_max (the
+ * Intel default for GPU-dominant apps, P@10496 / P@30503).  32 bytes. */
+typedef struct {
+  uint64_t q_base;        /* sum of quantised stretch at ratio_max           */
+  double   time_s;
+  double   energy_j;
+  uint64_t reserved;
+} magus_base;
+
+/* Per-config totals over traces: exact integer sums (uint64[16]) so that the
+ * cross-trace and cross-GPU reduction is order-free and bit-reproducible.
+ * The q sums are split into 32-bit limbs (q = hi*2^32 + lo per trace) so that
+ * each limb sum fits in 64 bits for any n_traces < 2^32, which also makes a
+ * plain NCCL uint64 sum exact. */
+enum {
+  MAGUS_TOT_N_TRACES = 0,
+  MAGUS_TOT_N_VIOL,
+  MAGUS_TOT_EVENTS,
+  MAGUS_TOT_HI_ROUNDS,
+  MAGUS_TOT_MSR_WRITES,
+  MAGUS_TOT_CHANGES,
+  MAGUS_TOT_MIN_DEC,
+  MAGUS_TOT_MIN_INT,
+  MAGUS_TOT_QMIN_LO,
+  MAGUS_TOT_QMIN_HI,
+  MAGUS_TOT_QMAX_LO,
+  MAGUS_TOT_QMAX_HI,
+  MAGUS_TOT_QBASE_LO,
+  MAGUS_TOT_QBASE_HI,
+  MAGUS_TOT_N_STEPS,     /* sum over traces of T                            */
+  MAGUS_TOT_RESERVED,
+  MAGUS_TOT_WORDS = 16
+};
+
+/* fp64 quantities derived from one config's integer totals (host-side,
+ * fixed operation order). */
+typedef struct {
+  double  energy_j;       /* fleet energy under MAGUS                         */
+  double  time_s;         /* fleet runtime under MAGUS                        */
+  double  base_energy_j;  /* fleet energy at ratio_max                        */
+  double  base_time_s;
+  double  saving;         /* 1 - energy_j / base_energy_j                     */
+  double  slowdown;       /* time_s / base_time_s - 1                         */
+  int64_t n_viol;         /* traces whose own slowdown exceeds the bound      */
+  int64_t n_traces;
+} magus_derived;
+
+/* ---- lifecycle -------------------------------------------------------- */
+
+/* Creates a context bound to CUDA `device`, enqueuing on `cuda_stream`
+ * (a cudaStream_t; NULL = legacy default stream).  Copies *plat. */
+magus_status magus_init(magus_ctx* out, int device, void* cuda_stream,
+                        const magus_platform* plat);
+magus_status magus_destroy(magus_ctx ctx);
+magus_status magus_set_stream(magus_ctx ctx, void* cuda_stream);
+const char*  magus_status_string(magus_status s);
+const char*  magus_last_error(magus_ctx ctx);
+int32_t      magus_abi_version(void);
+
+/* ---- presets (P@25197, P@44170, P@29320, P@29831, P@12253) ------------ */
+enum { MAGUS_POLICY_PAPER_DEFAULT = 0, MAGUS_POLICY_PAPER_PARETO = 1 };
+enum { MAGUS_PLATFORM_INTEL_A100 = 0, MAGUS_PLATFORM_INTEL_MAX1550 = 1 };
+magus_status magus_policy_preset(int32_t id, magus_policy* out);
+magus_status magus_platform_preset(int32_t id, magus_platform* out);
+/* SWEEP256: tau_inc {100,200,300,400} x tau_dec {-250,-500,-750,-1000} x
+ * t_hi {0.2,0.3,0.4,0.5} x W {4,6,10,16}; L = W, H = 10;
+ * index = iInc + 4*(iDec + 4*(iHi + 4*iW)).  paper_default = 165.
+ * FLEET64: same without the W axis, W = L = H = 10; paper_default = 37. */
+magus_status magus_grid_sweep256(magus_policy out[256]);
+magus_status magus_grid_fleet64(magus_policy out[64]);
+
+/* ---- the hot path ------------------------------------------------------ */
+
+/* Replays Alg. 1-3 over every interval of every trace for every config and
+ * scores the decisions with model M.
+ *   traces        device, fp32, TIME-MAJOR: sample t of trace n at
+ *                 traces[t*ld + n] (MB/s per interval).  NaN samples behave
+ *                 as "hold" (both Alg. 1 comparisons false).
+ *   n_traces      N >= 1;  n_steps T in [1, 2^24];  ld >= N.
+ *   params        HOST array of n_params (>= 1) configs.
+ *   out_summary   device [n_params][n_traces] or NULL.
+ *   out_base      device [n_traces] or NULL.
+ *   out_decisions device uint32 [n_params][ceil(T/32)][n_traces] or NULL:
+ *                 bit (t % 32) of word [c][t/32][n] is 1 iff dec[t] = ratio_min.
+ *                 (Time-blocked, trace-minor: each warp stores 128 contiguous
+ *                 bytes.)  Bits past T are 0.
+ *   out_totals    device uint64 [n_params][MAGUS_TOT_WORDS] or NULL.
+ * Asynchronous on the context stream. */
+magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t n_traces,
+                          int64_t n_steps, int64_t ld,
+                          const magus_policy* params, int32_t n_params,
+                          magus_summary* out_summary, magus_base* out_base,
+                          uint32_t* out_decisions, uint64_t* out_totals);
+
+/* End-to-end variant: every pointer is HOST memory (pinned or pageable).
+ * Stages traces host->device through context-owned buffers, runs
+ * magus_replay, copies the requested outputs back.  Synchronises. */
+magus_status magus_replay_host(magus_ctx ctx, const float* traces_host,
+                               int64_t n_traces, int64_t n_steps, int64_t ld,
+                               const magus_policy* params, int32_t n_params,
+                               magus_summary* summary_host,
+                               magus_base* base_host,
+                               uint32_t* decisions_host,
+                               uint64_t* totals_host);
+
+/* Derives the fp64 fleet quantities of one config from its integer totals
+ * (host memory, MAGUS_TOT_WORDS words) under the context's platform. */
+magus_status magus_totals_derive(magus_ctx ctx, const uint64_t* totals_host,
+                                 magus_derived* out);
+
+/* Picks the config of least fleet energy among those with n_viol == 0
+ * (the Sec. 6.4 choice on the energy/runtime front, P@44696, under the
+ * <5 % loss bound, P@1715).  Ties -> lowest index.  `totals` is DEVICE
+ * memory [n_params][MAGUS_TOT_WORDS] (already summed over ranks when
+ * sharded).  If no config is feasible returns MAGUS_ERR_NO_FEASIBLE with
+ * *best = argmin (n_viol, energy) and *best_row filled.  Synchronises. */
+magus_status magus_sweep_best(magus_ctx ctx, const uint64_t* totals,
+                              int32_t n_params, int32_t* best,
+                              magus_derived* best_row);
+
+/* ---- synthetic traces (input generator; gen/magus_gen.h) --------------- */
+enum { MAGUS_GEN_MIX = 0, MAGUS_GEN_ADVERSARIAL = 1 };
+/* Writes traces id0 .. id0+n_traces-1 of the seeded Markov phase model to
+ * device memory out[t*ld + i] (fp32, integer-valued MB/s).  Bit-identical to
+ * the host generator in gen/.  Asynchronous. */
+magus_status magus_gen_traces(magus_ctx ctx, uint64_t seed, int64_t id0,
+                              int64_t n_traces, int64_t n_steps, int64_t ld,
+                              int32_t kind, float* out);
+
+/* ---- options, instrumentation ------------------------------------------ */
+enum {
+  MAGUS_OPT_KERNEL = 0,       /* 0 auto, 1 reference (per-sample), 2 stream  */
+  MAGUS_OPT_SEGMENTS = 1,     /* 0 auto, else the number of time segments    */
+  MAGUS_OPT_TIMING = 2,       /* 1: record CUDA events around the main kernel */
+  MAGUS_OPT_WAVES = 3         /* target waves for auto segmentation (def. 4) */
+};
+magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value);
+
+typedef struct {
+  int64_t launches_total;     /* kernels launched by this context            */
+  int64_t main_launches;      /* replay-kernel launches timed (OPT_TIMING)   */
+  double  main_ms_total;      /* summed CUDA-event time of those launches    */
+  int64_t last_segments;      /* time segments used by the last replay       */
+  int64_t last_kernel;        /* 1 reference, 2 stream                       */
+  int64_t last_grid;          /* CTAs of the last main launch                */
+} magus_stats;
+/* Synchronises when timing is on (reads the events). */
+magus_status magus_get_stats(magus_ctx ctx, magus_stats* out);
+magus_status magus_reset_stats(magus_ctx ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MAGUS_H_ */

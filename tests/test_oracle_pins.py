@@ -1,0 +1,426 @@
+"""Pins of the CPU oracle against things other than itself (CPU only).
+
+Each test states what fixes the expected value: a hand-derived worked example
+(tests/golden/), a closed form, exact rational arithmetic, brute force, or an
+invariant the paper states.  P@N = byte offset into PAPER.md.
+"""
+from __future__ import annotations
+
+import glob
+import itertools
+import math
+import os
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+R_MIN, R_MAX = 8, 22
+
+
+# --------------------------------------------------------------------------
+# golden fixtures
+# --------------------------------------------------------------------------
+
+def _rle(s: str) -> list[int]:
+    out = []
+    for tok in s.split():
+        v, n = tok.split("*")
+        out += [int(v)] * int(n)
+    return out
+
+
+def _trace(spec: str, T: int) -> np.ndarray:
+    f = spec.split()
+    t = np.arange(T)
+    if f[0] == "const":
+        return np.full(T, float(f[1]), np.float32)
+    if f[0] == "step":
+        t0, a, b = int(f[1]), float(f[2]), float(f[3])
+        return np.where(t < t0, a, b).astype(np.float32)
+    if f[0] == "burst":
+        t0, w, base, peak = int(f[1]), int(f[2]), float(f[3]), float(f[4])
+        return np.where((t >= t0) & (t < t0 + w), peak, base).astype(np.float32)
+    if f[0] == "square":
+        lo, hi = float(f[1]), float(f[2])
+        return np.where(t % 2 == 0, lo, hi).astype(np.float32)
+    if f[0] == "values":
+        return np.array([float(v) for v in f[1:]], np.float32)
+    raise ValueError(spec)
+
+
+def _load_golden(path):
+    d = {}
+    for line in open(path):
+        line = line.strip()
+        if not line or line.startswith("#"):
+            continue
+        k, v = line.split(":", 1)
+        d[k.strip()] = v.strip()
+    return d
+
+
+GOLDEN_FILES = sorted(glob.glob(os.path.join(GOLDEN, "*.txt")))
+
+
+@pytest.mark.parametrize("path", GOLDEN_FILES, ids=[os.path.basename(p) for p in GOLDEN_FILES])
+@pytest.mark.parametrize("closed_form", [False, True])
+def test_golden_worked_examples(path, closed_form):
+    g = _load_golden(path)
+    T = int(g["T"])
+    x = _trace(g["trace"], T)
+    r = oracle.replay(x, oracle.policy(), want_dec=True, closed_form=closed_form)
+    assert r.dec[0, 0].tolist() == _rle(g["dec"])
+    assert r.hi[0, 0].tolist() == _rle(g["hi"])
+    s = r.summary[0, 0]
+    assert s["n_events"] == int(g["events"])
+    assert s["n_hi_rounds"] == int(g["hi_rounds"])
+    assert s["n_msr_writes"] == int(g["msr_writes"])
+    assert s["n_changes"] == int(g["changes"])
+
+
+# --------------------------------------------------------------------------
+# Alg. 1 (P@20631) and Alg. 2 (P@21063)
+# --------------------------------------------------------------------------
+
+def test_alg1_thresholds_and_ties():
+    # d = (ls[n] - ls[0]) / L with only the two ends read (lines 2-3)
+    z = [0.0] * 9
+    assert oracle.alg1(z + [2000.0], 10, 200, -500) == 0      # d == 200: not > 200
+    assert oracle.alg1(z + [2001.0], 10, 200, -500) == 1
+    assert oracle.alg1([5000.0] + z, 10, 200, -500) == 0      # d == -500: not < -500
+    assert oracle.alg1([5001.0] + z, 10, 200, -500) == -1
+    # interior values are ignored
+    assert oracle.alg1([0.0, 1e9, -1e9, 7.0, 2001.0], 10, 200, -500) == 1
+    # the divisor L scales d: 2001/1 > 1000? no; 2001/1 > 2000 yes
+    assert oracle.alg1([0.0, 2001.0], 1.0, 2000, -5000) == 1
+    assert oracle.alg1([0.0, 2001.0], 2.0, 2000, -5000) == 0
+    # increase wins when both thresholds are crossed (line 4 before line 6)
+    assert oracle.alg1([0.0, 100.0], 1.0, 5.0, 50.0) == 1
+    # NaN: both comparisons false -> 0 (reading R9)
+    assert oracle.alg1([0.0, float("nan")], 1.0, 5.0, -5.0) == 0
+
+
+def test_alg1_matches_exact_rational_away_from_rounding():
+    rng = np.random.default_rng(1)
+    for _ in range(2000):
+        a, b = (float(v) for v in rng.integers(0, 30000, 2))
+        L = float(rng.choice([1, 2, 4, 8, 10, 16]))
+        ti, td = float(rng.integers(50, 500)), -float(rng.integers(50, 1000))
+        d = Fraction(int(b) - int(a), int(L))
+        want = 1 if d > ti else (-1 if d < td else 0)
+        assert oracle.alg1([a, 3.0, b], L, ti, td) == want
+
+
+def test_alg2_exhaustive_vs_rational():
+    """s/n >= t_hi in fp64 (line 4 divides in floating point) equals the exact
+    rational comparison except where RN(s/n) lands exactly on t_hi, where the
+    fp64 '>=' must then be True."""
+    for H in range(1, 13):
+        for t_hi in (0.1, 0.2, 0.25, 0.3, 1 / 3, 0.4, 0.5, 0.7, 0.9, 1.0, 1.5):
+            for s in range(H + 1):
+                ls = [1] * s + [0] * (H - s)
+                got = oracle.alg2(ls, t_hi)
+                exact = Fraction(s, H) >= Fraction(t_hi)
+                rn_hits = float(Fraction(s, H)) == t_hi
+                assert got == (exact or rn_hits), (H, t_hi, s)
+    # the paper default: 4 of 10 rounds (P@25197 "0.4" with 10 zeros, P@24182)
+    assert oracle.alg2([1, 1, 1, 1, 0, 0, 0, 0, 0, 0], 0.4)
+    assert not oracle.alg2([1, 1, 1, 0, 0, 0, 0, 0, 0, 0], 0.4)
+    # order inside the FIFO does not matter (a sum)
+    for perm in set(itertools.permutations([1, 1, 1, 1, 0, 0, 0, 0, 0, 0])):
+        assert oracle.alg2(list(perm), 0.4)
+
+
+def test_alg2_fp64_boundary_fact():
+    # 1/10 rounds to the same double as 0.1 (which is above 1/10), so the
+    # fp64 predicate is True although the rational one is False.
+    assert float(Fraction(1, 10)) == 0.1 and Fraction(1, 10) < Fraction(0.1)
+    assert oracle.alg2([1] + [0] * 9, 0.1)
+    assert not oracle.alg2([0] * 10, 0.1)
+
+
+# --------------------------------------------------------------------------
+# Alg. 3 closed-form facts on longer traces
+# --------------------------------------------------------------------------
+
+def _replay(x, **pol):
+    return oracle.replay(np.asarray(x, np.float32), oracle.policy(**pol), want_dec=True)
+
+
+@pytest.mark.parametrize("value", [0.0, 1234.0, 24000.0])
+def test_constant_trace_constant_decision(value):
+    """F1 (north_star: 'a constant trace must give a constant decision')."""
+    r = _replay(np.full(5000, value))
+    s = r.summary[0, 0]
+    assert (r.dec == R_MAX).all()
+    assert s["n_events"] == s["n_msr_writes"] == s["n_changes"] == s["n_hi_rounds"] == 0
+    assert s["energy"] == r.base["energy"][0] and s["time"] == r.base["time"][0]
+    assert s["slowdown"] == 0.0
+
+
+@pytest.mark.parametrize("period", [1, 3, 9])
+def test_periodic_blind_spot(period):
+    """F2: a period dividing W-1 = 9 gives x[t] == x[t-9]: d = 0 always."""
+    vals = np.array([1000.0, 20000.0, 5000.0, 300.0, 9000.0, 100.0, 50.0, 7.0, 22000.0])[:period]
+    x = np.tile(vals, 4000 // period + 1)[:4000]
+    r = _replay(x)
+    assert (r.dec == R_MAX).all() and r.summary[0, 0]["n_events"] == 0
+
+
+@pytest.mark.parametrize("t0", [16, 37, 500])
+@pytest.mark.parametrize("W,H,t_hi", [(10, 10, 0.4), (4, 10, 0.4), (10, 10, 0.2), (16, 10, 0.5),
+                                      (6, 8, 0.3)])
+def test_step_down_latency(t0, W, H, t_hi):
+    """F3: a step at t0 >= W is detected in round t0 itself (the first window
+    that contains the new value), i.e. the decision switches after exactly
+    0 rounds; with k = min{s: s/H >= t_hi}, min holds for min(k, W-1) rounds."""
+    T = t0 + 60
+    x = np.where(np.arange(T) < t0, 20000.0, 1000.0)
+    r = _replay(x, W=W, H=H, t_hi=t_hi)
+    dec = r.dec[0, 0]
+    k = next(s for s in range(H + 2) if s > H or s / H >= t_hi)
+    assert (dec[:t0] == R_MAX).all()
+    n_min = min(k, W - 1)
+    assert (dec[t0:t0 + n_min] == R_MIN).all()
+    if k <= W - 1:  # enough events to trigger the frequent-transition rule
+        assert (dec[t0 + n_min:] == R_MAX).all()
+    else:
+        assert (dec[t0 + n_min:] == R_MIN).all()
+    assert r.summary[0, 0]["n_events"] == W - 1
+
+
+def test_oscillation_triggers_frequent_transition_rule():
+    """F6 / P@22101 / P@40055: rapid oscillation locks max via Alg. 2."""
+    T = 3000
+    x = np.where(np.arange(T) % 2 == 0, 1000.0, 20000.0)
+    r = _replay(x)
+    s = r.summary[0, 0]
+    assert (r.hi[0, 0][14:] == 1).all()
+    assert (r.dec[0, 0][14:] == R_MAX).all()
+    assert s["n_hi_rounds"] == T - 14
+
+
+# --------------------------------------------------------------------------
+# exhaustive: literal FIFO transcription == closed form; invariants
+# --------------------------------------------------------------------------
+
+def _all_traces(alphabet, T):
+    grid = np.array(list(itertools.product(alphabet, repeat=T)), dtype=np.float32)
+    return np.ascontiguousarray(grid.T)  # time-major [T, n]
+
+
+POLS = [dict(W=2, H=1, t_hi=1.0), dict(W=2, H=2, t_hi=0.5), dict(W=3, H=3, t_hi=0.6),
+        dict(W=4, H=5, t_hi=0.4), dict(W=5, H=4, t_hi=0.25), dict(W=3, H=10, t_hi=0.2),
+        dict(W=2, H=3, t_hi=2.0)]
+
+
+@pytest.mark.parametrize("pol", POLS, ids=[str(p) for p in POLS])
+def test_literal_equals_closed_form_exhaustive_binary(pol):
+    x = _all_traces([0.0, 30000.0], 14)
+    P = oracle.policy(**pol)
+    a = oracle.replay(x, P, want_dec=True)
+    b = oracle.replay(x, P, want_dec=True, closed_form=True)
+    assert np.array_equal(a.dec, b.dec) and np.array_equal(a.hi, b.hi)
+    assert np.array_equal(a.summary, b.summary)
+    _check_invariants(x, a, P[0])
+
+
+def test_literal_equals_closed_form_exhaustive_ternary():
+    x = _all_traces([0.0, 15000.0, 30000.0], 9)
+    for pol in POLS[:5]:
+        P = oracle.policy(**pol)
+        a = oracle.replay(x, P, want_dec=True)
+        b = oracle.replay(x, P, want_dec=True, closed_form=True)
+        assert np.array_equal(a.dec, b.dec) and np.array_equal(a.summary, b.summary)
+
+
+def _check_invariants(x, r, pol):
+    dec, hi, s = r.dec[0], r.hi[0], r.summary[0]
+    W = int(pol["W"])
+    assert np.isin(dec, [R_MIN, R_MAX]).all()                     # on the grid
+    assert (dec[:, :W] == R_MAX).all()                            # init at max (P@23755)
+    assert (dec[hi == 1] == R_MAX).all()                          # hi => max (P@22101)
+    assert (s["n_msr_writes"] >= s["n_changes"]).all()
+    assert (s["n_msr_writes"] >= s["n_hi_rounds"]).all()
+    changes = (dec[:, 1:] != dec[:, :-1]).sum(axis=1)
+    assert np.array_equal(changes, s["n_changes"])
+    assert np.array_equal((dec == R_MIN).sum(axis=1), s["n_min_dec"])
+    assert np.array_equal(s["n_min_int"], s["n_min_dec"] - (dec[:, -1] == R_MIN))
+    assert (s["slowdown"] >= 0.0).all()                           # exact (DESIGN 4.3)
+
+
+@pytest.mark.parametrize("kind", [gen.KIND_MIX, gen.KIND_ADVERSARIAL])
+def test_invariants_on_generator_traces(kind):
+    x = gen.gen_traces(gen.SEEDS[2], 48, 4000, kind=kind)
+    rng = np.random.default_rng(7)
+    rows = [dict(W=int(rng.choice([2, 4, 6, 10, 16, 33])), H=int(rng.choice([1, 5, 10, 20, 32, 64])),
+                 tau_inc=float(rng.choice([100, 200, 300, 400])),
+                 tau_dec=float(rng.choice([-250, -500, -1000])),
+                 t_hi=float(rng.choice([0.2, 0.3, 0.4, 0.5, 1.0]))) for _ in range(6)]
+    P = oracle.policies(rows)
+    a = oracle.replay(x, P, want_dec=True)
+    b = oracle.replay(x, P, want_dec=True, closed_form=True)
+    assert np.array_equal(a.dec, b.dec) and np.array_equal(a.summary, b.summary)
+    for c in range(len(rows)):
+        sub = oracle.OracleResult(a.summary[c:c + 1], a.base, a.dec[c:c + 1], a.hi[c:c + 1])
+        _check_invariants(x, sub, P[c])
+        hi_on = sub.summary[0]["n_hi_rounds"] > 0
+        k = next(s for s in range(rows[c]["H"] + 2) if s > rows[c]["H"] or s / rows[c]["H"] >= rows[c]["t_hi"])
+        assert (sub.summary[0]["n_events"][hi_on] >= k).all()
+
+
+# --------------------------------------------------------------------------
+# metamorphic relations (each follows from Alg. 1 reading only d's sign vs
+# the thresholds)
+# --------------------------------------------------------------------------
+
+def test_metamorphic_relations():
+    x = gen.gen_traces(gen.SEEDS[3], 32, 3000)
+    base = oracle.replay(x, oracle.policy(), want_dec=True)
+    for j in (-3, 2, 5):  # (x, tau) * 2^j: d scales exactly by 2^j
+        s = 2.0 ** j
+        r = oracle.replay(x * np.float32(s), oracle.policy(tau_inc=200 * s, tau_dec=-500 * s), want_dec=True)
+        assert np.array_equal(r.dec, base.dec)
+    for j in (1, 3):  # (L, tau) -> (2^j L, tau / 2^j)
+        s = 2.0 ** j
+        r = oracle.replay(x, oracle.policy(L=10 * s, tau_inc=200 / s, tau_dec=-500 / s), want_dec=True)
+        assert np.array_equal(r.dec, base.dec)
+    # integer shift of an integer-valued trace: differences unchanged
+    r = oracle.replay(x + np.float32(777), oracle.policy(), want_dec=True)
+    assert np.array_equal(r.dec, base.dec)
+    # negation with mirrored thresholds: same events and hi sequence
+    r = oracle.replay(-x, oracle.policy(tau_inc=500, tau_dec=-200), want_dec=True)
+    assert np.array_equal(r.hi, base.hi)
+    assert np.array_equal(r.summary["n_events"], base.summary["n_events"])
+
+
+# --------------------------------------------------------------------------
+# model M: exact arithmetic, closed forms, brute force
+# --------------------------------------------------------------------------
+
+def test_model_exact_stretch_power_of_two_platform():
+    """bw_max = 16384 at r_max = 16, r_min = 8 -> B_min = 2^13 exactly, so the
+    stretch of x = 3 * 2^13 at min is exactly 2 (q = 2 * 2^24)."""
+    plat = oracle.platform(r_min=8, r_max=16, bw_max=16384.0, beta=0.5, p_other=100.0,
+                           p_unc_min=0.0, p_unc_max=64.0)
+    T = 8
+    x = np.full(T, 3 * 8192.0, np.float32)
+    dec = np.full(T, 8, np.int32)                # min from round 0 on
+    s, b = oracle.account(x, dec, plat)
+    assert s["n_min_int"] == T - 1 and s["q_min"] == (T - 1) * 2 * 2 ** 24
+    # at max the capacity is 2^14: stretch 0.5 = 2^23 units per interval
+    assert b["q_base"] == T * 2 ** 23 and s["q_max"] == 2 ** 23
+    dt, beta = Fraction(0.2), Fraction(1, 2)
+    # exact rational model, then compare within a few ulp of the fp64 result
+    t_min = dt * (T - 1) + dt * beta * (T - 1) * 2
+    t_max = dt * 1 + dt * beta * Fraction(1, 2)
+    e = 164 * t_max + 100 * t_min
+    assert math.isclose(s["energy"], float(e), rel_tol=4e-16)
+    assert math.isclose(s["time"], float(t_min + t_max), rel_tol=4e-16)
+
+
+def test_model_no_stretch_saving_matches_paper_calibration():
+    """All-min schedule with x below every capacity: saving = 1 - P_min/P_max
+    over the min intervals; with the Fig. 2 calibration (82 W of 300 W,
+    P@12253) this is the paper's 'up to 27 %' headline scale (P@1715)."""
+    T = 10001
+    x = np.full(T, 500.0, np.float32)
+    dec = np.full(T, R_MIN, np.int32)
+    s, b = oracle.account(x, dec)
+    saving = 1.0 - s["energy"] / b["energy"]
+    exact = 1 - Fraction(300 + 218 * (T - 1), 300 * T)
+    assert math.isclose(saving, float(exact), rel_tol=1e-12)
+    assert abs(saving - 82 / 300) < 1e-4 and s["slowdown"] == 0.0
+
+
+def test_model_slowdown_nonnegative_and_zero_without_stretch():
+    x = gen.gen_traces(gen.SEEDS[1], 64, 2000)
+    r = oracle.replay(x, oracle.policy())
+    assert (r.summary["slowdown"] >= 0).all()
+    xs = np.minimum(x, np.float32(11000.0))      # below B_min = 11636.36
+    r2 = oracle.replay(xs, oracle.policy())
+    assert (r2.summary["slowdown"] == 0.0).all()
+    assert (r2.summary["q_min"] == 0).all() and (r2.base["q_base"] == 0).all()
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_bruteforce_energy_lower_bound(seed):
+    """north_star: on tiny traces the exhaustive minimum over all {min,max}^T
+    schedules is a lower bound MAGUS never beats (also under the slowdown
+    bound whenever MAGUS itself is feasible)."""
+    T = 13
+    rng = np.random.default_rng(seed)
+    x = rng.choice([300.0, 900.0, 12000.0, 15000.0, 23000.0], size=T).astype(np.float32)
+    plat = oracle.platform(bound=0.02)
+    r = oracle.replay(x, oracle.policy(W=3, H=3, t_hi=0.6), plat, want_dec=True)
+    e_magus = r.summary[0, 0]["energy"]
+    feasible = r.summary[0, 0]["slowdown"] <= 0.02
+    best = best_feasible = math.inf
+    for bits in range(1 << T):
+        dec = np.array([R_MIN if (bits >> t) & 1 else R_MAX for t in range(T)], np.int32)
+        s, _ = oracle.account(x, dec, plat)
+        best = min(best, s["energy"])
+        if s["slowdown"] <= 0.02:
+            best_feasible = min(best_feasible, s["energy"])
+    assert best <= e_magus * (1 + 1e-12)
+    if feasible:
+        assert best_feasible <= e_magus * (1 + 1e-12)
+
+
+def test_totals_exact_and_sum_of_parts():
+    x = gen.gen_traces(gen.SEEDS[2], 200, 3000)
+    r = oracle.replay(x, oracle.policy())
+    w, f = oracle.totals(r.summary[0], r.base, 3000)
+    s = r.summary[0]
+    assert w[0] == 200 and w[1] == s["viol"].sum() and w[2] == s["n_events"].sum()
+    qmin = sum(int(v) for v in s["q_min"])
+    assert int(w[8]) + (int(w[9]) << 32) == qmin
+    # fleet energy vs the exactly rounded sum of per-trace energies
+    assert math.isclose(f[0], math.fsum(s["energy"].tolist()), rel_tol=1e-12)
+    assert math.isclose(oracle.energy_sum(s), math.fsum(s["energy"].tolist()), rel_tol=1e-15)
+    assert math.isclose(f[2], math.fsum(r.base["energy"].tolist()), rel_tol=1e-12)
+
+
+def test_sweep_best_rules():
+    assert oracle.sweep_best([0, 0, 1], [5.0, 4.0, 1.0]) == (1, True)
+    assert oracle.sweep_best([0, 0], [4.0, 4.0]) == (0, True)         # ties -> lowest
+    assert oracle.sweep_best([2, 1, 1], [1.0, 3.0, 2.0]) == (2, False)  # infeasible
+
+
+def test_digest_definition():
+    """digest = sum_w word_w * (mix64(w) | 1) mod 2^64."""
+    x = gen.gen_traces(gen.SEEDS[1], 8, 1000)
+    r = oracle.replay(x, oracle.policy(), want_dec=True)
+    words = oracle.decision_words(r.dec[0], R_MIN)
+
+    def mix64(z):
+        m = (1 << 64) - 1
+        z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & m
+        z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & m
+        return z ^ (z >> 31)
+    for n in range(8):
+        d = sum(int(wd) * (mix64(w) | 1) for w, wd in enumerate(words[n])) % (1 << 64)
+        assert d == int(r.summary[0, n]["digest"])
+
+
+def test_degenerate_shapes():
+    # T < W: no MDFS round at all
+    r = _replay(np.array([1.0, 50000.0, 0.0], np.float32))
+    assert (r.dec == R_MAX).all() and r.summary[0, 0]["n_msr_writes"] == 0
+    # T == W: still no round; T == W + 1: exactly one
+    r = _replay(np.r_[np.zeros(10), 30000.0].astype(np.float32))
+    assert r.summary[0, 0]["n_events"] == 1 and r.summary[0, 0]["n_msr_writes"] == 1
+    # NaN samples behave as "hold"
+    x = np.full(40, 1000.0, np.float32)
+    x[20] = np.nan
+    r = _replay(x)
+    assert (r.dec == R_MAX).all() and r.summary[0, 0]["n_events"] == 0
+    with pytest.raises(ValueError):
+        oracle.replay(np.zeros(10, np.float32), oracle.policy(W=1))
+    with pytest.raises(ValueError):
+        oracle.replay(np.zeros(10, np.float32), oracle.policy(t_hi=0.0))
