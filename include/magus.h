@@ -243,6 +243,27 @@ magus_status magus_gen_traces(magus_ctx ctx, uint64_t seed, int64_t id0,
                               int64_t n_traces, int64_t n_steps, int64_t ld,
                               int32_t kind, float* out);
 
+/* ---- diagnostics of the host precompute (no GPU needed) ----------------- */
+/* The stream kernel never divides: Alg. 1's "d = delta/L > tau_inc" becomes
+ * "delta > delta_inc" with delta_inc the largest double whose RN quotient by L
+ * does not exceed tau_inc (exact because RN(delta/L) is monotone in delta);
+ * likewise "delta < delta_dec"; Alg. 2's "s/H >= t_hi" becomes s >= k_hi
+ * (k_hi = H+1: never).  Model M's "RN(x * (1/B_l)) > 1" becomes the float
+ * comparison x > x_stretch_l. */
+typedef struct {
+  double  delta_inc;
+  double  delta_dec;
+  int32_t k_hi;
+  int32_t reserved;
+} magus_policy_consts;
+typedef struct {
+  float   x_stretch_min, x_stretch_max;
+  double  inv_cap_min, inv_cap_max;   /* 1 / B_l in (MB/s)^-1 */
+  double  p_min_w, p_max_w;           /* model-M power at ratio_min / max */
+} magus_platform_consts;
+magus_status magus_policy_inspect(const magus_policy* p, magus_policy_consts* out);
+magus_status magus_platform_inspect(const magus_platform* p, magus_platform_consts* out);
+
 /* ---- options, instrumentation ------------------------------------------ */
 enum {
   MAGUS_OPT_KERNEL = 0,       /* 0 auto, 1 reference (per-sample), 2 stream  */

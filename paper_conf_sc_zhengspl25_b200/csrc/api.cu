@@ -1,0 +1,662 @@
+// api.cu -- libmagus C-ABI (include/magus.h): validation, per-config host
+// precompute, scratch management, kernel dispatch, totals, sweep choice.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <string>
+#include <utility>
+#include <vector>
+
+#include "magus_internal.h"
+
+using namespace magus;
+
+struct magus_ctx_s {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  magus_platform plat{};
+  DevPlatform dplat{};
+  std::string err;
+  int sms = 148;
+  // options
+  int64_t opt_kernel = 0, opt_segments = 0, opt_timing = 0, opt_waves = 4;
+  // device scratch
+  void* scratch = nullptr;
+  size_t scratch_bytes = 0;
+  // policy upload cache
+  std::vector<magus_policy> last_params;
+  void* pol_dev = nullptr;
+  size_t pol_dev_bytes = 0;
+  void* pol_host = nullptr;  // pinned staging
+  size_t pol_host_bytes = 0;
+  cudaEvent_t pol_copied = nullptr;
+  std::vector<std::pair<std::pair<int, int>, std::vector<int32_t>>> groups;  // (W,H) -> configs
+  std::vector<int64_t> group_offsets;                                        // into cidx
+  // e2e staging (device)
+  void* stage_dev = nullptr;
+  size_t stage_bytes = 0;
+  // stats
+  int64_t launches = 0, main_launches = 0, last_segments = 0, last_kernel = 0, last_grid = 0;
+  double main_ms = 0.0;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> pending;
+  std::vector<cudaEvent_t> event_pool;
+  std::map<std::pair<int, int>, int> ctas_cache;
+  PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+};
+
+namespace {
+
+magus_status fail(magus_ctx ctx, magus_status st, const char* fmt, ...) {
+  if (ctx) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    std::vsnprintf(buf, sizeof(buf), fmt, ap);
+    va_end(ap);
+    ctx->err = buf;
+  }
+  return st;
+}
+
+magus_status cuda_fail(magus_ctx ctx, cudaError_t e, const char* what) {
+  return fail(ctx, MAGUS_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+#define CK(call)                                   \
+  do {                                             \
+    cudaError_t e_ = (call);                       \
+    if (e_ != cudaSuccess) return cuda_fail(ctx, e_, #call); \
+  } while (0)
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+magus_status ensure_scratch(magus_ctx ctx, size_t bytes) {
+  if (bytes <= ctx->scratch_bytes) return MAGUS_OK;
+  // the stream may still use the old buffer
+  CK(cudaStreamSynchronize(ctx->stream));
+  if (ctx->scratch) cudaFree(ctx->scratch);
+  ctx->scratch = nullptr;
+  ctx->scratch_bytes = 0;
+  const size_t want = align_up(bytes + bytes / 8, 1 << 20);
+  cudaError_t e = cudaMalloc(&ctx->scratch, want);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(ctx, MAGUS_ERR_OOM, "scratch allocation of %zu bytes failed", want);
+  }
+  ctx->scratch_bytes = want;
+  return MAGUS_OK;
+}
+
+cudaEvent_t take_event(magus_ctx ctx) {
+  if (!ctx->event_pool.empty()) {
+    cudaEvent_t e = ctx->event_pool.back();
+    ctx->event_pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+
+bool same_params(const std::vector<magus_policy>& a, const magus_policy* b, int32_t n) {
+  if ((int32_t)a.size() != n) return false;
+  return std::memcmp(a.data(), b, sizeof(magus_policy) * (size_t)n) == 0;
+}
+
+// Uploads DevPolicy[C] + config index lists of the (W,H) groups.
+magus_status upload_policies(magus_ctx ctx, const magus_policy* params, int32_t C) {
+  if (same_params(ctx->last_params, params, C) && ctx->pol_dev) return MAGUS_OK;
+  std::vector<DevPolicy> dp((size_t)C);
+  std::map<std::pair<int, int>, std::vector<int32_t>> g;
+  for (int32_t c = 0; c < C; ++c) {
+    dp[c] = make_dev_policy(params[c]);
+    g[{params[c].window, params[c].history}].push_back(c);
+  }
+  ctx->groups.assign(g.begin(), g.end());
+  ctx->group_offsets.clear();
+  std::vector<int32_t> cidx;
+  for (auto& kv : ctx->groups) {
+    ctx->group_offsets.push_back((int64_t)cidx.size());
+    cidx.insert(cidx.end(), kv.second.begin(), kv.second.end());
+  }
+  const size_t pol_bytes = align_up(sizeof(DevPolicy) * (size_t)C, 256);
+  const size_t need = pol_bytes + sizeof(int32_t) * cidx.size();
+  if (ctx->pol_copied) CK(cudaEventSynchronize(ctx->pol_copied));  // pinned buffer reuse
+  if (need > ctx->pol_dev_bytes) {
+    CK(cudaStreamSynchronize(ctx->stream));
+    if (ctx->pol_dev) cudaFree(ctx->pol_dev);
+    ctx->pol_dev = nullptr;
+    CK(cudaMalloc(&ctx->pol_dev, need));
+    ctx->pol_dev_bytes = need;
+  }
+  if (need > ctx->pol_host_bytes) {
+    if (ctx->pol_host) cudaFreeHost(ctx->pol_host);
+    ctx->pol_host = nullptr;
+    CK(cudaMallocHost(&ctx->pol_host, need));
+    ctx->pol_host_bytes = need;
+  }
+  std::memcpy(ctx->pol_host, dp.data(), sizeof(DevPolicy) * (size_t)C);
+  std::memcpy((char*)ctx->pol_host + pol_bytes, cidx.data(), sizeof(int32_t) * cidx.size());
+  CK(cudaMemcpyAsync(ctx->pol_dev, ctx->pol_host, need, cudaMemcpyHostToDevice, ctx->stream));
+  if (!ctx->pol_copied) CK(cudaEventCreateWithFlags(&ctx->pol_copied, cudaEventDisableTiming));
+  CK(cudaEventRecord(ctx->pol_copied, ctx->stream));
+  ctx->last_params.assign(params, params + C);
+  return MAGUS_OK;
+}
+
+const DevPolicy* dev_policies(magus_ctx ctx) { return (const DevPolicy*)ctx->pol_dev; }
+const int32_t* dev_cidx(magus_ctx ctx, int64_t off) {
+  const size_t pol_bytes = align_up(sizeof(DevPolicy) * ctx->last_params.size(), 256);
+  return (const int32_t*)((const char*)ctx->pol_dev + pol_bytes) + off;
+}
+
+int ctas_per_sm(magus_ctx ctx, int W, int H) {
+  auto key = std::make_pair(W, H);
+  auto it = ctx->ctas_cache.find(key);
+  if (it != ctx->ctas_cache.end()) return it->second;
+  int v = stream_ctas_per_sm(W, H);
+  ctx->ctas_cache[key] = v;
+  return v;
+}
+
+magus_status encode_tmap(magus_ctx ctx, CUtensorMap* map, const float* x, int64_t N, int64_t T,
+                         int64_t ld) {
+  if (!ctx->encode) {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    CK(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
+    if (!fn || q != cudaDriverEntryPointSuccess)
+      return fail(ctx, MAGUS_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+    ctx->encode = (PFN_cuTensorMapEncodeTiled_v12000)fn;
+  }
+  cuuint64_t dims[2] = {(cuuint64_t)N, (cuuint64_t)T};
+  cuuint64_t strides[1] = {(cuuint64_t)ld * 4};
+  cuuint32_t box[2] = {128, 32};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = ctx->encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)x, dims, strides, box,
+                           estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(ctx, MAGUS_ERR_CUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  return MAGUS_OK;
+}
+
+magus_status validate_replay(magus_ctx ctx, const float* traces, int64_t N, int64_t T, int64_t ld,
+                             const magus_policy* params, int32_t C) {
+  if (!traces) return fail(ctx, MAGUS_ERR_INVALID_ARG, "traces is NULL");
+  if (N < 1 || N > ((int64_t)1 << 31) - 1) return fail(ctx, MAGUS_ERR_INVALID_ARG, "n_traces %lld out of range", (long long)N);
+  if (T < 1 || T > kMaxSteps) return fail(ctx, MAGUS_ERR_INVALID_ARG, "n_steps %lld not in [1, 2^24]", (long long)T);
+  if (ld < N) return fail(ctx, MAGUS_ERR_INVALID_ARG, "ld %lld < n_traces %lld", (long long)ld, (long long)N);
+  if (!params || C < 1) return fail(ctx, MAGUS_ERR_INVALID_ARG, "no params");
+  char msg[256];
+  for (int32_t c = 0; c < C; ++c)
+    if (!validate_policy(params[c], msg, sizeof msg))
+      return fail(ctx, MAGUS_ERR_INVALID_ARG, "params[%d]: %s", c, msg);
+  return MAGUS_OK;
+}
+
+}  // namespace
+
+namespace magus {
+
+static double u128_to_double(unsigned __int128 v) { return (double)v; }
+
+void derive_totals(const DevPlatform& p, const uint64_t* w, magus_derived* out) {
+  const uint64_t NT = w[MAGUS_TOT_N_STEPS];
+  const uint64_t mint = w[MAGUS_TOT_MIN_INT];
+  const unsigned __int128 qmin =
+      ((unsigned __int128)w[MAGUS_TOT_QMIN_HI] << 32) + (unsigned __int128)w[MAGUS_TOT_QMIN_LO];
+  const unsigned __int128 qmax =
+      ((unsigned __int128)w[MAGUS_TOT_QMAX_HI] << 32) + (unsigned __int128)w[MAGUS_TOT_QMAX_LO];
+  const unsigned __int128 qbase =
+      ((unsigned __int128)w[MAGUS_TOT_QBASE_HI] << 32) + (unsigned __int128)w[MAGUS_TOT_QBASE_LO];
+  const double ch = (double)w[MAGUS_TOT_CHANGES];
+  const double time_max = p.dt * (double)(NT - mint) + p.cQ * u128_to_double(qmax);
+  const double time_min = p.dt * (double)mint + p.cQ * u128_to_double(qmin);
+  const double time = (p.dt * (double)NT + p.cQ * u128_to_double(qmin + qmax)) + p.t_sw * ch;
+  const double energy = (p.P_max * time_max + p.P_min * time_min) + p.e_sw * ch;
+  const double base_time = p.dt * (double)NT + p.cQ * u128_to_double(qbase);
+  const double base_energy = p.P_max * base_time;
+  out->energy_j = energy;
+  out->time_s = time;
+  out->base_energy_j = base_energy;
+  out->base_time_s = base_time;
+  out->saving = 1.0 - energy / base_energy;
+  out->slowdown = time / base_time - 1.0;
+  out->n_viol = (int64_t)w[MAGUS_TOT_N_VIOL];
+  out->n_traces = (int64_t)w[MAGUS_TOT_N_TRACES];
+}
+
+}  // namespace magus
+
+extern "C" {
+
+int32_t magus_abi_version(void) { return MAGUS_ABI_VERSION; }
+
+const char* magus_status_string(magus_status s) {
+  switch (s) {
+    case MAGUS_OK: return "ok";
+    case MAGUS_ERR_INVALID_ARG: return "invalid argument";
+    case MAGUS_ERR_NOT_INITIALIZED: return "not initialized";
+    case MAGUS_ERR_CUDA: return "CUDA error";
+    case MAGUS_ERR_NCCL: return "NCCL error";
+    case MAGUS_ERR_OOM: return "out of device memory";
+    case MAGUS_ERR_UNSUPPORTED: return "unsupported";
+    case MAGUS_ERR_NO_FEASIBLE: return "no feasible config";
+  }
+  return "unknown status";
+}
+
+const char* magus_last_error(magus_ctx ctx) { return ctx ? ctx->err.c_str() : "NULL context"; }
+
+magus_status magus_policy_preset(int32_t id, magus_policy* out) {
+  if (!out) return MAGUS_ERR_INVALID_ARG;
+  magus_policy p;
+  p.window = 10;        // reading R4
+  p.history = 10;       // P@24182
+  p.deriv_len = 10.0;   // reading R4: L = W
+  p.tau_dec = -500.0;   // P@25197 "500", signed per reading R1
+  p.t_hi = 0.4;         // P@25197
+  if (id == MAGUS_POLICY_PAPER_DEFAULT) p.tau_inc = 200.0;       // P@25197 (Sec. 3.3)
+  else if (id == MAGUS_POLICY_PAPER_PARETO) p.tau_inc = 300.0;   // P@44170 (Sec. 6.4)
+  else return MAGUS_ERR_INVALID_ARG;
+  *out = p;
+  return MAGUS_OK;
+}
+
+magus_status magus_platform_preset(int32_t id, magus_platform* out) {
+  if (!out) return MAGUS_ERR_INVALID_ARG;
+  magus_platform p;
+  p.ratio_min = 8;            // 0.8 GHz (P@29320 / P@29831)
+  if (id == MAGUS_PLATFORM_INTEL_A100) p.ratio_max = 22;          // 2.2 GHz, P@29320
+  else if (id == MAGUS_PLATFORM_INTEL_MAX1550) p.ratio_max = 25;  // 2.5 GHz, P@29831
+  else return MAGUS_ERR_INVALID_ARG;
+  p.dt_s = 0.2;               // P@44789
+  p.bw_max_mbs = 32000.0;     // model-M assumption
+  p.beta = 1.0;               // model-M assumption
+  p.p_other_w = 218.0;        // 118 W CPU at min uncore (Fig. 2) + 100 W board (assumption)
+  p.p_unc_min_w = 0.0;
+  p.p_unc_max_w = 82.0;       // Fig. 2: 200 W -> 120 W (P@12253)
+  p.e_switch_j = 0.0;         // "negligible" (P@27899)
+  p.t_switch_s = 0.0;
+  p.slowdown_bound = 0.05;    // P@1715
+  *out = p;
+  return MAGUS_OK;
+}
+
+static const double kGridInc[4] = {100.0, 200.0, 300.0, 400.0};
+static const double kGridDec[4] = {-250.0, -500.0, -750.0, -1000.0};
+static const double kGridHi[4] = {0.2, 0.3, 0.4, 0.5};
+static const int32_t kGridW[4] = {4, 6, 10, 16};
+
+magus_status magus_grid_sweep256(magus_policy out[256]) {
+  if (!out) return MAGUS_ERR_INVALID_ARG;
+  for (int iW = 0; iW < 4; ++iW)
+    for (int iHi = 0; iHi < 4; ++iHi)
+      for (int iDec = 0; iDec < 4; ++iDec)
+        for (int iInc = 0; iInc < 4; ++iInc) {
+          magus_policy& p = out[iInc + 4 * (iDec + 4 * (iHi + 4 * iW))];
+          p.window = kGridW[iW];
+          p.history = 10;
+          p.deriv_len = (double)kGridW[iW];
+          p.tau_inc = kGridInc[iInc];
+          p.tau_dec = kGridDec[iDec];
+          p.t_hi = kGridHi[iHi];
+        }
+  return MAGUS_OK;
+}
+
+magus_status magus_grid_fleet64(magus_policy out[64]) {
+  if (!out) return MAGUS_ERR_INVALID_ARG;
+  for (int iHi = 0; iHi < 4; ++iHi)
+    for (int iDec = 0; iDec < 4; ++iDec)
+      for (int iInc = 0; iInc < 4; ++iInc) {
+        magus_policy& p = out[iInc + 4 * (iDec + 4 * iHi)];
+        p.window = 10;
+        p.history = 10;
+        p.deriv_len = 10.0;
+        p.tau_inc = kGridInc[iInc];
+        p.tau_dec = kGridDec[iDec];
+        p.t_hi = kGridHi[iHi];
+      }
+  return MAGUS_OK;
+}
+
+magus_status magus_policy_inspect(const magus_policy* p, magus_policy_consts* out) {
+  char msg[256];
+  if (!p || !out || !validate_policy(*p, msg, sizeof msg)) return MAGUS_ERR_INVALID_ARG;
+  const DevPolicy d = make_dev_policy(*p);
+  out->delta_inc = d.d_inc;
+  out->delta_dec = d.d_dec;
+  out->k_hi = d.k;
+  out->reserved = 0;
+  return MAGUS_OK;
+}
+
+magus_status magus_platform_inspect(const magus_platform* p, magus_platform_consts* out) {
+  char msg[256];
+  if (!p || !out || !validate_platform(*p, msg, sizeof msg)) return MAGUS_ERR_INVALID_ARG;
+  const DevPlatform d = make_dev_platform(*p);
+  out->x_stretch_min = d.xthr_min;
+  out->x_stretch_max = d.xthr_max;
+  out->inv_cap_min = d.invB_min;
+  out->inv_cap_max = d.invB_max;
+  out->p_min_w = d.P_min;
+  out->p_max_w = d.P_max;
+  return MAGUS_OK;
+}
+
+magus_status magus_init(magus_ctx* out, int device, void* cuda_stream, const magus_platform* plat) {
+  if (!out || !plat) return MAGUS_ERR_INVALID_ARG;
+  *out = nullptr;
+  char msg[256];
+  if (!validate_platform(*plat, msg, sizeof msg)) return MAGUS_ERR_INVALID_ARG;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
+    cudaGetLastError();
+    return MAGUS_ERR_CUDA;
+  }
+  cudaDeviceProp prop;
+  if (cudaGetDeviceProperties(&prop, device) != cudaSuccess) return MAGUS_ERR_CUDA;
+  if (prop.major != 10) return MAGUS_ERR_UNSUPPORTED;  // built for sm_100a only
+  magus_ctx ctx = new magus_ctx_s();
+  ctx->device = device;
+  ctx->stream = (cudaStream_t)cuda_stream;
+  ctx->plat = *plat;
+  ctx->dplat = make_dev_platform(*plat);
+  ctx->sms = prop.multiProcessorCount;
+  *out = ctx;
+  return MAGUS_OK;
+}
+
+magus_status magus_destroy(magus_ctx ctx) {
+  if (!ctx) return MAGUS_ERR_INVALID_ARG;
+  {
+    DeviceGuard dg(ctx->device);
+    cudaStreamSynchronize(ctx->stream);
+    if (ctx->scratch) cudaFree(ctx->scratch);
+    if (ctx->pol_dev) cudaFree(ctx->pol_dev);
+    if (ctx->pol_host) cudaFreeHost(ctx->pol_host);
+    if (ctx->stage_dev) cudaFree(ctx->stage_dev);
+    if (ctx->pol_copied) cudaEventDestroy(ctx->pol_copied);
+    for (auto& pr : ctx->pending) {
+      cudaEventDestroy(pr.first);
+      cudaEventDestroy(pr.second);
+    }
+    for (auto e : ctx->event_pool) cudaEventDestroy(e);
+  }
+  delete ctx;
+  return MAGUS_OK;
+}
+
+magus_status magus_set_stream(magus_ctx ctx, void* cuda_stream) {
+  if (!ctx) return MAGUS_ERR_INVALID_ARG;
+  ctx->stream = (cudaStream_t)cuda_stream;
+  return MAGUS_OK;
+}
+
+magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value) {
+  if (!ctx) return MAGUS_ERR_INVALID_ARG;
+  switch (key) {
+    case MAGUS_OPT_KERNEL:
+      if (value < 0 || value > 2) return fail(ctx, MAGUS_ERR_INVALID_ARG, "kernel option %lld", (long long)value);
+      ctx->opt_kernel = value;
+      return MAGUS_OK;
+    case MAGUS_OPT_SEGMENTS:
+      if (value < 0) return fail(ctx, MAGUS_ERR_INVALID_ARG, "segments < 0");
+      ctx->opt_segments = value;
+      return MAGUS_OK;
+    case MAGUS_OPT_TIMING:
+      ctx->opt_timing = value ? 1 : 0;
+      return MAGUS_OK;
+    case MAGUS_OPT_WAVES:
+      if (value < 1 || value > 64) return fail(ctx, MAGUS_ERR_INVALID_ARG, "waves not in [1, 64]");
+      ctx->opt_waves = value;
+      return MAGUS_OK;
+  }
+  return fail(ctx, MAGUS_ERR_INVALID_ARG, "unknown option %d", key);
+}
+
+magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t N, int64_t T, int64_t ld,
+                          const magus_policy* params, int32_t C, magus_summary* out_summary,
+                          magus_base* out_base, uint32_t* out_decisions, uint64_t* out_totals) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  magus_status st = validate_replay(ctx, traces, N, T, ld, params, C);
+  if (st != MAGUS_OK) return st;
+  DeviceGuard dg(ctx->device);
+  cudaGetLastError();
+
+  // kernel choice
+  bool all_stream = true;
+  for (int32_t c = 0; c < C; ++c)
+    all_stream = all_stream && stream_supported(params[c].window, params[c].history);
+  const bool tma_ok = ((uintptr_t)traces % 16 == 0) && (ld % 4 == 0);
+  int kernel = (int)ctx->opt_kernel;
+  if (kernel == 0) kernel = (all_stream && tma_ok) ? 2 : 1;
+  if (kernel == 2 && !(all_stream && tma_ok))
+    return fail(ctx, MAGUS_ERR_UNSUPPORTED,
+                "stream kernel needs W in [2,33], H in [1,32], 16-B aligned traces and ld %% 4 == 0");
+
+  st = upload_policies(ctx, params, C);
+  if (st != MAGUS_OK) return st;
+
+  // scratch: summaries / base when the caller does not want them but totals need them
+  const int64_t nw = (T + 31) / 32;
+  int64_t nseg = 1, seg_len = ((T + 31) / 32) * 32;
+  if (kernel == 2) {
+    const int64_t ngroups = (N + 127) / 128;
+    if (ctx->opt_segments > 0) {
+      nseg = ctx->opt_segments;
+    } else {
+      int per_sm = 1 << 30;
+      for (auto& g : ctx->groups) per_sm = std::min(per_sm, ctas_per_sm(ctx, g.first.first, g.first.second));
+      if (per_sm < 1) per_sm = 1;
+      const int64_t slots = (int64_t)ctx->sms * per_sm * ctx->opt_waves;
+      nseg = std::max<int64_t>(1, (slots + ngroups * C - 1) / (ngroups * C));
+    }
+    seg_len = ((T + nseg - 1) / nseg + 31) / 32 * 32;
+    const int64_t min_len = 512;  // keeps the halo re-read below ~6 %
+    if (ctx->opt_segments == 0 && seg_len < min_len) seg_len = std::min<int64_t>(min_len, ((T + 31) / 32) * 32);
+    nseg = (T + seg_len - 1) / seg_len;
+  }
+  const size_t sum_bytes = (out_summary || !out_totals) ? 0 : align_up(sizeof(magus_summary) * (size_t)(N * C), 256);
+  const size_t base_bytes = (out_base || !out_totals) ? 0 : align_up(sizeof(magus_base) * (size_t)N, 256);
+  const size_t nrec = (kernel == 2) ? (size_t)C * (size_t)nseg * (size_t)N : 0;
+  const size_t rec_bytes = align_up(nrec * 4, 256) * 8 + align_up(nrec * 8, 256) * 7;
+  st = ensure_scratch(ctx, sum_bytes + base_bytes + rec_bytes + 256);
+  if (st != MAGUS_OK) return st;
+  char* sp = (char*)ctx->scratch;
+  magus_summary* summ = out_summary;
+  if (!summ && out_totals) { summ = (magus_summary*)sp; sp += sum_bytes; }
+  magus_base* base = out_base;
+  if (!base && out_totals) { base = (magus_base*)sp; sp += base_bytes; }
+
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  if (ctx->opt_timing) {
+    ev0 = take_event(ctx);
+    ev1 = take_event(ctx);
+    CK(cudaEventRecord(ev0, ctx->stream));
+  }
+  int launched = 0;
+  if (kernel == 1) {
+    int r = launch_reference(ctx->stream, traces, N, T, ld, dev_policies(ctx), C, ctx->dplat, summ,
+                             base, out_decisions);
+    if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "reference kernel launch");
+    launched += r;
+    ctx->last_grid = (N * C + 127) / 128;
+    if (ctx->opt_timing) CK(cudaEventRecord(ev1, ctx->stream));
+  } else {
+    SegRecords rec;
+    uint32_t** u32s[8] = {&rec.ev, &rec.hi, &rec.msr, &rec.ch, &rec.mdec, &rec.mint, &rec.flags, &rec.apos};
+    for (auto p : u32s) { *p = (uint32_t*)sp; sp += align_up(nrec * 4, 256); }
+    unsigned long long** u64s[7] = {&rec.qmin, &rec.qmax, &rec.qbase, &rec.dig, &rec.pqmin, &rec.pqmax, &rec.pdig};
+    for (auto p : u64s) { *p = (unsigned long long*)sp; sp += align_up(nrec * 8, 256); }
+    CUtensorMap map;
+    st = encode_tmap(ctx, &map, traces, N, T, ld);
+    if (st != MAGUS_OK) return st;
+    int64_t grid_total = 0;
+    for (size_t gi = 0; gi < ctx->groups.size(); ++gi) {
+      auto& g = ctx->groups[gi];
+      int grid = 0;
+      int r = launch_stream(ctx->stream, &map, N, T, dev_policies(ctx), dev_cidx(ctx, ctx->group_offsets[gi]),
+                            (int32_t)g.second.size(), g.first.first, g.first.second, ctx->dplat, nseg,
+                            seg_len, rec, out_decisions, nw * N, &grid);
+      if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "stream kernel launch");
+      launched += r;
+      grid_total += grid;
+    }
+    ctx->last_grid = grid_total;
+    if (ctx->opt_timing) CK(cudaEventRecord(ev1, ctx->stream));
+    int r = launch_fixup(ctx->stream, N, T, C, ctx->dplat, nseg, seg_len, rec, summ, base, out_decisions);
+    if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "fixup kernel launch");
+    launched += r;
+  }
+  if (out_totals) {
+    int r = launch_totals(ctx->stream, summ, base, N, T, C, out_totals);
+    if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "totals kernel launch");
+    launched += r;
+  }
+  if (ctx->opt_timing) ctx->pending.push_back({ev0, ev1});
+  ctx->launches += launched;
+  ctx->last_segments = nseg;
+  ctx->last_kernel = kernel;
+  return MAGUS_OK;
+}
+
+magus_status magus_replay_host(magus_ctx ctx, const float* traces_host, int64_t N, int64_t T,
+                               int64_t ld, const magus_policy* params, int32_t C,
+                               magus_summary* summary_host, magus_base* base_host,
+                               uint32_t* decisions_host, uint64_t* totals_host) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  magus_status st = validate_replay(ctx, traces_host, N, T, ld, params, C);
+  if (st != MAGUS_OK) return st;
+  DeviceGuard dg(ctx->device);
+  const int64_t ldd = (N + 3) / 4 * 4;
+  const int64_t nw = (T + 31) / 32;
+  const size_t x_bytes = align_up(sizeof(float) * (size_t)(ldd * T), 256);
+  const size_t s_bytes = summary_host ? align_up(sizeof(magus_summary) * (size_t)(N * C), 256) : 0;
+  const size_t b_bytes = base_host ? align_up(sizeof(magus_base) * (size_t)N, 256) : 0;
+  const size_t d_bytes = decisions_host ? align_up(sizeof(uint32_t) * (size_t)(C * nw * N), 256) : 0;
+  const size_t t_bytes = totals_host ? align_up(sizeof(uint64_t) * (size_t)(C * MAGUS_TOT_WORDS), 256) : 0;
+  const size_t need = x_bytes + s_bytes + b_bytes + d_bytes + t_bytes;
+  if (need > ctx->stage_bytes) {
+    CK(cudaStreamSynchronize(ctx->stream));
+    if (ctx->stage_dev) cudaFree(ctx->stage_dev);
+    ctx->stage_dev = nullptr;
+    ctx->stage_bytes = 0;
+    cudaError_t e = cudaMalloc(&ctx->stage_dev, need);
+    if (e != cudaSuccess) { cudaGetLastError(); return fail(ctx, MAGUS_ERR_OOM, "staging allocation failed"); }
+    ctx->stage_bytes = need;
+  }
+  char* p = (char*)ctx->stage_dev;
+  float* xd = (float*)p; p += x_bytes;
+  magus_summary* sd = summary_host ? (magus_summary*)p : nullptr; p += s_bytes;
+  magus_base* bd = base_host ? (magus_base*)p : nullptr; p += b_bytes;
+  uint32_t* dd = decisions_host ? (uint32_t*)p : nullptr; p += d_bytes;
+  uint64_t* td = totals_host ? (uint64_t*)p : nullptr;
+  CK(cudaMemcpy2DAsync(xd, ldd * 4, traces_host, ld * 4, N * 4, T, cudaMemcpyHostToDevice, ctx->stream));
+  st = magus_replay(ctx, xd, N, T, ldd, params, C, sd, bd, dd, td);
+  if (st != MAGUS_OK) return st;
+  if (summary_host) CK(cudaMemcpyAsync(summary_host, sd, sizeof(magus_summary) * N * C, cudaMemcpyDeviceToHost, ctx->stream));
+  if (base_host) CK(cudaMemcpyAsync(base_host, bd, sizeof(magus_base) * N, cudaMemcpyDeviceToHost, ctx->stream));
+  if (decisions_host) CK(cudaMemcpyAsync(decisions_host, dd, sizeof(uint32_t) * C * nw * N, cudaMemcpyDeviceToHost, ctx->stream));
+  if (totals_host) CK(cudaMemcpyAsync(totals_host, td, sizeof(uint64_t) * C * MAGUS_TOT_WORDS, cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  return MAGUS_OK;
+}
+
+magus_status magus_totals_derive(magus_ctx ctx, const uint64_t* totals_host, magus_derived* out) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  if (!totals_host || !out) return fail(ctx, MAGUS_ERR_INVALID_ARG, "NULL argument");
+  derive_totals(ctx->dplat, totals_host, out);
+  return MAGUS_OK;
+}
+
+magus_status magus_sweep_best(magus_ctx ctx, const uint64_t* totals, int32_t C, int32_t* best,
+                              magus_derived* best_row) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  if (!totals || C < 1 || !best) return fail(ctx, MAGUS_ERR_INVALID_ARG, "bad sweep_best arguments");
+  DeviceGuard dg(ctx->device);
+  std::vector<uint64_t> h((size_t)C * MAGUS_TOT_WORDS);
+  CK(cudaMemcpyAsync(h.data(), totals, h.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  std::vector<magus_derived> d((size_t)C);
+  for (int32_t c = 0; c < C; ++c) derive_totals(ctx->dplat, h.data() + (size_t)c * MAGUS_TOT_WORDS, &d[c]);
+  int32_t b = -1;
+  for (int32_t c = 0; c < C; ++c)
+    if (d[c].n_viol == 0 && (b < 0 || d[c].energy_j < d[b].energy_j)) b = c;
+  magus_status st = MAGUS_OK;
+  if (b < 0) {
+    st = MAGUS_ERR_NO_FEASIBLE;
+    b = 0;
+    for (int32_t c = 1; c < C; ++c)
+      if (d[c].n_viol < d[b].n_viol || (d[c].n_viol == d[b].n_viol && d[c].energy_j < d[b].energy_j)) b = c;
+    ctx->err = "no config keeps every trace within the slowdown bound";
+  }
+  *best = b;
+  if (best_row) *best_row = d[b];
+  return st;
+}
+
+magus_status magus_gen_traces(magus_ctx ctx, uint64_t seed, int64_t id0, int64_t N, int64_t T,
+                              int64_t ld, int32_t kind, float* out) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  if (!out || N < 1 || T < 1 || ld < N || id0 < 0 || (kind != MAGUS_GEN_MIX && kind != MAGUS_GEN_ADVERSARIAL))
+    return fail(ctx, MAGUS_ERR_INVALID_ARG, "bad gen arguments");
+  DeviceGuard dg(ctx->device);
+  if (launch_gen(ctx->stream, seed, id0, N, T, ld, kind, out) < 0)
+    return cuda_fail(ctx, cudaGetLastError(), "gen kernel launch");
+  ctx->launches += 1;
+  return MAGUS_OK;
+}
+
+magus_status magus_get_stats(magus_ctx ctx, magus_stats* out) {
+  if (!ctx || !out) return MAGUS_ERR_INVALID_ARG;
+  DeviceGuard dg(ctx->device);
+  for (auto& pr : ctx->pending) {
+    CK(cudaEventSynchronize(pr.second));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, pr.first, pr.second));
+    ctx->main_ms += ms;
+    ctx->main_launches += 1;
+    ctx->event_pool.push_back(pr.first);
+    ctx->event_pool.push_back(pr.second);
+  }
+  ctx->pending.clear();
+  out->launches_total = ctx->launches;
+  out->main_launches = ctx->main_launches;
+  out->main_ms_total = ctx->main_ms;
+  out->last_segments = ctx->last_segments;
+  out->last_kernel = ctx->last_kernel;
+  out->last_grid = ctx->last_grid;
+  return MAGUS_OK;
+}
+
+magus_status magus_reset_stats(magus_ctx ctx) {
+  if (!ctx) return MAGUS_ERR_INVALID_ARG;
+  magus_stats tmp;
+  magus_status st = magus_get_stats(ctx, &tmp);  // drains pending events
+  ctx->launches = 0;
+  ctx->main_launches = 0;
+  ctx->main_ms = 0.0;
+  return st;
+}
+
+}  // extern "C"

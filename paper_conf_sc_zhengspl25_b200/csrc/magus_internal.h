@@ -1,0 +1,89 @@
+// magus_internal.h -- device-side parameter blocks and launch plumbing shared
+// by the libmagus translation units (NOT part of the C-ABI).
+#pragma once
+
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "../../include/magus.h"
+
+namespace magus {
+
+// Stretch metering of model M: the per-interval stretch
+// sigma = max(0, x/B_l - 1) is capped at 2^15 intervals and metered in units
+// of 2^-24 interval, so every accumulation is an exact integer sum.
+constexpr double kQScale = 16777216.0;                 // 2^24
+constexpr double kQCapScaled = 549755813888.0;         // 2^15 * 2^24 = 2^39
+constexpr int64_t kMaxSteps = int64_t(1) << 24;       // keeps sum q < 2^63
+
+// Per-config constants, precomputed on the host (precompute.cpp).
+struct DevPolicy {
+  // Alg. 1 literal form (reference kernel): d = delta / L
+  double L, tau_inc, tau_dec;
+  // Alg. 1 inverted form (stream kernel): delta > d_inc  <=> RN(delta/L) > tau_inc
+  //                                        delta < d_dec  <=> RN(delta/L) < tau_dec
+  double d_inc, d_dec;
+  // Alg. 2 literal form: (double)s / (double)H >= t_hi
+  double t_hi;
+  // Alg. 2 inverted form: s >= k  (k = H+1: never)
+  int32_t W, H, k, pad;
+};
+
+// Platform / model-M constants.
+struct DevPlatform {
+  int32_t r_min, r_max;
+  // literal form (reference kernel): r = x * invB; r > 1 -> s = r - 1 ...
+  double invB_min, invB_max;
+  // inverted form (stream kernel): x > xthr <=> RN(x*invB) > 1 ; r24 = x*invB24
+  float xthr_min, xthr_max;
+  double invB24_min, invB24_max;
+  // finalisation (fp64, fixed order)
+  double dt, cQ, P_max, P_min, e_sw, t_sw, bound;
+};
+
+// Segment records of the stream kernel, struct-of-arrays [C][nseg][N].
+struct SegRecords {
+  uint32_t *ev, *hi, *msr, *ch, *mdec, *mint, *flags, *apos;
+  unsigned long long *qmin, *qmax, *qbase, *dig, *pqmin, *pqmax, *pdig;
+};
+enum : uint32_t { kFlagHypMin = 1u, kFlagSeen = 2u, kFlagVa = 4u, kFlagLastMin = 8u };
+
+// Host precompute (precompute.cpp); returns false + message on invalid input.
+bool validate_policy(const magus_policy& p, char* msg, size_t n);
+bool validate_platform(const magus_platform& p, char* msg, size_t n);
+DevPolicy make_dev_policy(const magus_policy& p);
+DevPlatform make_dev_platform(const magus_platform& p);
+double invert_inc(double L, double tau_inc);
+double invert_dec(double L, double tau_dec);
+float stretch_threshold(double invB);
+
+// Launchers (each returns the number of kernels launched, or -1 on error).
+
+int launch_reference(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,
+                     const DevPolicy* pol_dev, int32_t C, const DevPlatform& plat,
+                     magus_summary* out_summary, magus_base* out_base, uint32_t* out_dec);
+
+bool stream_supported(int32_t W, int32_t H);
+// Stream kernel over the nc configs listed in cidx_dev (global indices; all
+// share (W, H)).  Records / decisions are indexed by the global config index.
+int launch_stream(cudaStream_t s, const void* tmap /* CUtensorMap, host copy */, int64_t N,
+                  int64_t T, const DevPolicy* pol_dev, const int32_t* cidx_dev, int32_t nc,
+                  int32_t W, int32_t H, const DevPlatform& plat, int64_t nseg, int64_t seg_len,
+                  const SegRecords& rec, uint32_t* out_dec, int64_t dec_cstride, int* grid_out);
+int stream_ctas_per_sm(int32_t W, int32_t H);
+
+// Resolves the segment carries of all C configs and writes the summaries.
+int launch_fixup(cudaStream_t s, int64_t N, int64_t T, int32_t C, const DevPlatform& plat,
+                 int64_t nseg, int64_t seg_len, const SegRecords& rec, magus_summary* out_summary,
+                 magus_base* out_base, uint32_t* out_dec);
+
+int launch_totals(cudaStream_t s, const magus_summary* summary, const magus_base* base, int64_t N,
+                  int64_t T, int32_t C, uint64_t* totals);
+
+int launch_gen(cudaStream_t s, uint64_t seed, int64_t id0, int64_t N, int64_t T, int64_t ld,
+               int32_t kind, float* out);
+
+// host-side derivation of fleet quantities (api.cu)
+void derive_totals(const DevPlatform& p, const uint64_t* w, magus_derived* out);
+
+}  // namespace magus

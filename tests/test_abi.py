@@ -1,0 +1,133 @@
+"""C-ABI surface checks that need no GPU: the library loads, exports every
+function include/magus.h declares, and its host-only calls behave."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared():
+    src = open(os.path.join(ROOT, "include", "magus.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(magus_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol():
+    import paper_conf_sc_zhengspl25_b200 as m
+    names = _declared()
+    assert "magus_replay" in names and "magus_sweep_best" in names and "magus_init" in names
+    lib = ctypes.CDLL(m.LIB_PATH)
+    missing = [n for n in names if not hasattr(lib, n)]
+    assert not missing, missing
+    assert set(m.EXPORTED) == set(names)
+    assert m.abi_version() == 1
+
+
+def test_presets_cite_the_paper_values():
+    import paper_conf_sc_zhengspl25_b200 as m
+    d = m.policy_preset(m.POLICY_PAPER_DEFAULT)
+    assert (d.window, d.history, d.deriv_len, d.tau_inc, d.tau_dec, d.t_hi) == (10, 10, 10.0, 200.0, -500.0, 0.4)
+    assert m.policy_preset(m.POLICY_PAPER_PARETO).tau_inc == 300.0
+    a = m.platform_preset(m.PLATFORM_INTEL_A100)
+    assert (a.ratio_min, a.ratio_max, a.dt_s, a.p_unc_max_w, a.slowdown_bound) == (8, 22, 0.2, 82.0, 0.05)
+    assert m.platform_preset(m.PLATFORM_INTEL_MAX1550).ratio_max == 25
+    with pytest.raises(m.MagusError):
+        m.policy_preset(7)
+
+
+def test_grids_index_convention():
+    import paper_conf_sc_zhengspl25_b200 as m
+    g = m.grid_sweep256()
+    d = g[165]
+    assert (d.window, d.tau_inc, d.tau_dec, d.t_hi) == (10, 200.0, -500.0, 0.4)
+    assert g[166].tau_inc == 300.0
+    seen = {(p.window, p.tau_inc, p.tau_dec, p.t_hi) for p in g}
+    assert len(seen) == 256 and all(p.deriv_len == p.window and p.history == 10 for p in g)
+    f = m.grid_fleet64()
+    assert (f[37].tau_inc, f[37].tau_dec, f[37].t_hi) == (200.0, -500.0, 0.4) and f[38].tau_inc == 300.0
+
+
+def test_init_without_gpu_fails_cleanly():
+    import paper_conf_sc_zhengspl25_b200 as m
+    try:
+        import torch
+        if torch.cuda.is_available():
+            pytest.skip("GPU present")
+    except ImportError:
+        pass
+    h = ctypes.c_void_p()
+    p = m.platform_preset()
+    st = m._lib.magus_init(ctypes.byref(h), 0, None, ctypes.byref(p))
+    assert st == m.ERR_CUDA and not h.value
+
+
+def test_null_context_is_rejected():
+    import paper_conf_sc_zhengspl25_b200 as m
+    assert m._lib.magus_replay(None, None, 1, 1, 1, None, 1, None, None, None, None) == m.ERR_NOT_INITIALIZED
+    assert m._lib.magus_last_error(None) == b"NULL context"
+    assert m._lib.magus_status_string(m.ERR_NO_FEASIBLE) == b"no feasible config"
+
+
+def test_ptxas_report_has_no_spills_on_the_hot_kernel():
+    log = open(os.path.join(ROOT, "paper_conf_sc_zhengspl25_b200", "build", "ptxas.log")).read()
+    blocks = re.split(r"Compiling entry function", log)
+    hot = [b for b in blocks if "stream_kernelILi10ELi10E" in b]
+    assert hot, "stream_kernel<10,10> missing from the build"
+    assert "0 bytes spill stores" in hot[0]
+
+
+def test_binding_structs_match_header_sizes():
+    import paper_conf_sc_zhengspl25_b200 as m
+    assert ctypes.sizeof(m.Policy) == 40 and ctypes.sizeof(m.Platform) == 80
+    assert m.SUMMARY_DT.itemsize == 104 and m.BASE_DT.itemsize == 32
+    assert np.dtype(np.uint64).itemsize * m.TOT_WORDS == 128
+
+
+def _nextafter(x, d):
+    return float(np.nextafter(np.float64(x), np.float64(d)))
+
+
+def test_threshold_inversion_equals_literal_division():
+    """delta > delta_inc <=> RN(delta/L) > tau_inc (Alg. 1 l.3-4), checked at
+    delta_inc and its neighbours, for awkward L and tau (Python's float
+    division is IEEE round-to-nearest, like the paper's C++)."""
+    import paper_conf_sc_zhengspl25_b200 as m
+    rng = np.random.default_rng(3)
+    cases = [(10.0, 200.0, -500.0), (3.0, 0.1, -0.7), (7.0, 1 / 3, -2 / 3), (0.3, 17.0, -19.0),
+             (1e-300, 1e300, -1e300), (1e300, 1e-300, -1e-300), (5.0, 0.0, 0.0), (2.0, -3.0, 4.0)]
+    cases += [(float(rng.uniform(0.01, 100)), float(rng.uniform(-1e4, 1e4)), float(rng.uniform(-1e4, 1e4)))
+              for _ in range(300)]
+    for L, ti, td in cases:
+        c = m.policy_inspect(m.make_policy(W=10, L=L, tau_inc=ti, tau_dec=td))
+        for base in (c["delta_inc"], c["delta_dec"], ti * L, td * L, 0.0, -0.0):
+            for d in (_nextafter(_nextafter(base, -np.inf), -np.inf), _nextafter(base, -np.inf), base,
+                      _nextafter(base, np.inf), _nextafter(_nextafter(base, np.inf), np.inf)):
+                assert (d > c["delta_inc"]) == (d / L > ti), (L, ti, d)
+                assert (d < c["delta_dec"]) == (d / L < td), (L, td, d)
+        for d in (np.inf, -np.inf):
+            assert (d > c["delta_inc"]) == (d / L > ti) and (d < c["delta_dec"]) == (d / L < td)
+
+
+def test_k_hi_matches_alg2():
+    import paper_conf_sc_zhengspl25_b200 as m
+    for H in (1, 3, 7, 10, 32, 64):
+        for t_hi in (0.1, 0.2, 0.3, 0.4, 0.5, 1 / 3, 0.99, 1.0, 1.01, 5.0):
+            k = m.policy_inspect(m.make_policy(H=H, t_hi=t_hi))["k_hi"]
+            want = next((s for s in range(H + 1) if s / H >= t_hi), H + 1)
+            assert k == want
+
+
+def test_stretch_threshold_equals_literal_predicate():
+    import paper_conf_sc_zhengspl25_b200 as m
+    for bw in (32000.0, 16384.0, 12345.678, 1e-3, 3e38):
+        p = m.platform_preset()
+        p.bw_max_mbs = bw
+        c = m.platform_inspect(p)
+        for thr, inv in ((c["x_stretch_min"], c["inv_cap_min"]), (c["x_stretch_max"], c["inv_cap_max"])):
+            f = np.float32(thr)
+            for x in (np.nextafter(f, np.float32(-np.inf)), f, np.nextafter(f, np.float32(np.inf))):
+                assert (x > f) == (float(x) * inv > 1.0)
