@@ -102,7 +102,7 @@ struct Window {  // compile-time H: ripple-carry bit-sliced counter (6 bits, H <
     uint32_t c[6] = {0, 0, 0, 0, 0, 0};
 #pragma unroll
     for (int j = 1; j <= H; ++j) {
-      uint32_t b = __funnelshift_l(Ep, E, j);
+      uint32_t b = __funnelshift_lc(Ep, E, j);  // clamps: j = 32 -> Ep
 #pragma unroll
       for (int l = 0; l < 6; ++l) {
         const uint32_t t = c[l] & b;
@@ -139,7 +139,7 @@ struct Window<0> {  // runtime H <= 32
   static __device__ __forceinline__ uint32_t ge(uint32_t E, uint32_t Ep, int H, const KMask& km) {
     uint32_t c[6] = {0, 0, 0, 0, 0, 0};
     for (int j = 1; j <= H; ++j) {
-      uint32_t b = __funnelshift_l(Ep, E, j);
+      uint32_t b = __funnelshift_lc(Ep, E, j);  // clamps: j = 32 -> Ep
 #pragma unroll
       for (int l = 0; l < 6; ++l) {
         const uint32_t t = c[l] & b;

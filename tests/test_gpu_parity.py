@@ -43,7 +43,7 @@ def to_oracle_policies(pols):
 
 def run_gpu(ctx, x_np, pols, kernel, segments=0, ld=None, decisions=True):
     T, N = x_np.shape
-    ld = N if ld is None else ld
+    ld = (N + 3) // 4 * 4 if ld is None else ld      # TMA needs a 16-B row pitch
     xd = torch.zeros((T, ld), dtype=torch.float32, device="cuda:0")
     xd[:, :N] = torch.from_numpy(x_np).cuda()
     ctx.set_option(magus.OPT_KERNEL, kernel)
