@@ -29,6 +29,8 @@ struct magus_ctx_s {
   // device scratch
   void* scratch = nullptr;
   size_t scratch_bytes = 0;
+  uint64_t work_sig = 0;   // layout of the fused kernel's counters in scratch
+  uint32_t epoch = 0;      // per-replay tag of the segment status words
   // policy upload cache
   std::vector<magus_policy> last_params;
   void* pol_dev = nullptr;
@@ -90,6 +92,7 @@ size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
 
 magus_status ensure_scratch(magus_ctx ctx, size_t bytes) {
   if (bytes <= ctx->scratch_bytes) return MAGUS_OK;
+  ctx->work_sig = 0;
   // the stream may still use the old buffer
   CK(cudaStreamSynchronize(ctx->stream));
   if (ctx->scratch) cudaFree(ctx->scratch);
@@ -102,6 +105,7 @@ magus_status ensure_scratch(magus_ctx ctx, size_t bytes) {
     return fail(ctx, MAGUS_ERR_OOM, "scratch allocation of %zu bytes failed", want);
   }
   ctx->scratch_bytes = want;
+  CK(cudaMemsetAsync(ctx->scratch, 0, want, ctx->stream));  // counters start at zero
   return MAGUS_OK;
 }
 
@@ -457,7 +461,6 @@ magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t N, int64_t
   st = upload_policies(ctx, params, C);
   if (st != MAGUS_OK) return st;
 
-  // scratch: summaries / base when the caller does not want them but totals need them
   const int64_t nw = (T + 31) / 32;
   int64_t nseg = 1, seg_len = ((T + 31) / 32) * 32;
   if (kernel == 2) {
@@ -476,62 +479,89 @@ magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t N, int64_t
     if (ctx->opt_segments == 0 && seg_len < min_len) seg_len = std::min<int64_t>(min_len, ((T + 31) / 32) * 32);
     nseg = (T + seg_len - 1) / seg_len;
   }
-  const size_t sum_bytes = (out_summary || !out_totals) ? 0 : align_up(sizeof(magus_summary) * (size_t)(N * C), 256);
-  const size_t base_bytes = (out_base || !out_totals) ? 0 : align_up(sizeof(magus_base) * (size_t)N, 256);
-  const size_t nrec = (kernel == 2) ? (size_t)C * (size_t)nseg * (size_t)N : 0;
-  const size_t rec_bytes = align_up(nrec * 4, 256) * 8 + align_up(nrec * 8, 256) * 7;
-  st = ensure_scratch(ctx, sum_bytes + base_bytes + rec_bytes + 256);
-  if (st != MAGUS_OK) return st;
-  char* sp = (char*)ctx->scratch;
-  magus_summary* summ = out_summary;
-  if (!summ && out_totals) { summ = (magus_summary*)sp; sp += sum_bytes; }
-  magus_base* base = out_base;
-  if (!base && out_totals) { base = (magus_base*)sp; sp += base_bytes; }
-
+  const int64_t ngroups = (N + 127) / 128;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   if (ctx->opt_timing) {
     ev0 = take_event(ctx);
     ev1 = take_event(ctx);
-    CK(cudaEventRecord(ev0, ctx->stream));
   }
   int launched = 0;
   if (kernel == 1) {
+    // the reference kernel writes summaries directly; totals need them
+    const size_t sum_bytes = (out_summary || !out_totals) ? 0 : align_up(sizeof(magus_summary) * (size_t)(N * C), 256);
+    const size_t base_bytes = (out_base || !out_totals) ? 0 : align_up(sizeof(magus_base) * (size_t)N, 256);
+    st = ensure_scratch(ctx, sum_bytes + base_bytes + 256);
+    if (st != MAGUS_OK) return st;
+    ctx->work_sig = 0;  // scratch reused: the stream path must re-zero its counters
+    char* sp = (char*)ctx->scratch;
+    magus_summary* summ = out_summary;
+    if (!summ && out_totals) { summ = (magus_summary*)sp; sp += sum_bytes; }
+    magus_base* base = out_base;
+    if (!base && out_totals) base = (magus_base*)sp;
+    if (ctx->opt_timing) CK(cudaEventRecord(ev0, ctx->stream));
     int r = launch_reference(ctx->stream, traces, N, T, ld, dev_policies(ctx), C, ctx->dplat, summ,
                              base, out_decisions);
     if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "reference kernel launch");
     launched += r;
     ctx->last_grid = (N * C + 127) / 128;
     if (ctx->opt_timing) CK(cudaEventRecord(ev1, ctx->stream));
+    if (out_totals) {
+      r = launch_totals(ctx->stream, summ, base, N, T, C, out_totals);
+      if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "totals kernel launch");
+      launched += r;
+    }
   } else {
-    SegRecords rec;
-    uint32_t** u32s[8] = {&rec.ev, &rec.hi, &rec.msr, &rec.ch, &rec.mdec, &rec.mint, &rec.flags, &rec.apos};
-    for (auto p : u32s) { *p = (uint32_t*)sp; sp += align_up(nrec * 4, 256); }
-    unsigned long long** u64s[7] = {&rec.qmin, &rec.qmax, &rec.qbase, &rec.dig, &rec.pqmin, &rec.pqmax, &rec.pdig};
-    for (auto p : u64s) { *p = (unsigned long long*)sp; sp += align_up(nrec * 8, 256); }
+    // scratch of the fused kernel: counters + accumulators (zero, self-cleaning)
+    // followed by the epoch-tagged segment status words
+    const size_t off_arrive = 256;
+    const size_t off_tarrive = off_arrive + align_up(4 * (size_t)(C * ngroups), 256);
+    const size_t off_tacc = off_tarrive + align_up(4 * (size_t)C, 256);
+    const size_t off_acc = off_tacc + align_up(8 * 13 * (size_t)C, 256);
+    const size_t off_status = off_acc + align_up(8 * (size_t)kAccFields * (size_t)(C * N), 256);
+    const size_t total = off_status + align_up(4 * (size_t)(C * nseg) * (size_t)N, 256);
+    st = ensure_scratch(ctx, total);
+    if (st != MAGUS_OK) return st;
+    const uint64_t sig = ((uint64_t)C * 1000003ULL + (uint64_t)N) * 1000033ULL + (uint64_t)nseg + 1;
+    if (sig != ctx->work_sig) {
+      CK(cudaMemsetAsync(ctx->scratch, 0, off_status, ctx->stream));
+      ctx->work_sig = sig;
+    }
+    if (++ctx->epoch >= (1u << 29)) {
+      CK(cudaMemsetAsync(ctx->scratch, 0, total, ctx->stream));
+      ctx->epoch = 1;
+    }
+    char* sp = (char*)ctx->scratch;
+    StreamWork wk;
+    wk.ticket = (uint32_t*)sp;
+    wk.done = (uint32_t*)sp + 1;
+    wk.arrive = (uint32_t*)(sp + off_arrive);
+    wk.tarrive = (uint32_t*)(sp + off_tarrive);
+    wk.tacc = (unsigned long long*)(sp + off_tacc);
+    wk.acc = (unsigned long long*)(sp + off_acc);
+    wk.status = (uint32_t*)(sp + off_status);
+    wk.epoch = ctx->epoch;
+    wk.summary = out_summary;
+    wk.base = out_base;
+    wk.dec = out_decisions;
+    wk.dec_cstride = nw * N;
+    wk.totals = out_totals;
     CUtensorMap map;
     st = encode_tmap(ctx, &map, traces, N, T, ld);
     if (st != MAGUS_OK) return st;
+    if (ctx->opt_timing) CK(cudaEventRecord(ev0, ctx->stream));
     int64_t grid_total = 0;
     for (size_t gi = 0; gi < ctx->groups.size(); ++gi) {
       auto& g = ctx->groups[gi];
       int grid = 0;
       int r = launch_stream(ctx->stream, &map, N, T, dev_policies(ctx), dev_cidx(ctx, ctx->group_offsets[gi]),
                             (int32_t)g.second.size(), g.first.first, g.first.second, ctx->dplat, nseg,
-                            seg_len, rec, out_decisions, nw * N, &grid);
+                            seg_len, wk, &grid);
       if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "stream kernel launch");
       launched += r;
       grid_total += grid;
     }
     ctx->last_grid = grid_total;
     if (ctx->opt_timing) CK(cudaEventRecord(ev1, ctx->stream));
-    int r = launch_fixup(ctx->stream, N, T, C, ctx->dplat, nseg, seg_len, rec, summ, base, out_decisions);
-    if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "fixup kernel launch");
-    launched += r;
-  }
-  if (out_totals) {
-    int r = launch_totals(ctx->stream, summ, base, N, T, C, out_totals);
-    if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "totals kernel launch");
-    launched += r;
   }
   if (ctx->opt_timing) ctx->pending.push_back({ev0, ev1});
   ctx->launches += launched;

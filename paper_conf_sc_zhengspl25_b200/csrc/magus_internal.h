@@ -41,12 +41,26 @@ struct DevPlatform {
   double dt, cQ, P_max, P_min, e_sw, t_sw, bound;
 };
 
-// Segment records of the stream kernel, struct-of-arrays [C][nseg][N].
-struct SegRecords {
-  uint32_t *ev, *hi, *msr, *ch, *mdec, *mint, *flags, *apos;
-  unsigned long long *qmin, *qmax, *qbase, *dig, *pqmin, *pqmax, *pdig;
+// Work/scratch block of the fused stream kernel (kernels_stream.cu).  The
+// counters and accumulators are zero at allocation and self-cleaning (the
+// last user of each resets it); the segment status words are tagged with a
+// per-replay epoch, so nothing needs a memset between replays.
+constexpr int kAccFields = 10;  // ev hi msr ch mdec mint qmin qmax qbase dig
+struct StreamWork {
+  uint32_t* ticket;              // [1] launch-order work ticket
+  uint32_t* done;                // [1] finished CTAs of the launch
+  uint32_t* status;              // [C][nseg][N] epoch<<3 | last_min<<2 | seen<<1 | 1
+  unsigned long long* acc;       // [C][kAccFields][N] segment sums
+  uint32_t* arrive;              // [C][ngroups] finished segments
+  unsigned long long* tacc;      // [C][13] totals under construction
+  uint32_t* tarrive;             // [C] finished groups
+  uint32_t epoch;
+  magus_summary* summary;        // [C][N] or NULL
+  magus_base* base;              // [N] or NULL
+  uint32_t* dec;                 // [C][nw][N] or NULL
+  int64_t dec_cstride;           // nw * N
+  uint64_t* totals;              // [C][16] or NULL
 };
-enum : uint32_t { kFlagHypMin = 1u, kFlagSeen = 2u, kFlagVa = 4u, kFlagLastMin = 8u };
 
 // Host precompute (precompute.cpp); returns false + message on invalid input.
 bool validate_policy(const magus_policy& p, char* msg, size_t n);
@@ -64,18 +78,13 @@ int launch_reference(cudaStream_t s, const float* x, int64_t N, int64_t T, int64
                      magus_summary* out_summary, magus_base* out_base, uint32_t* out_dec);
 
 bool stream_supported(int32_t W, int32_t H);
-// Stream kernel over the nc configs listed in cidx_dev (global indices; all
-// share (W, H)).  Records / decisions are indexed by the global config index.
+// Fused stream kernel over the nc configs listed in cidx_dev (global indices;
+// all share (W, H)): replay + carry look-back + finalisation + totals.
 int launch_stream(cudaStream_t s, const void* tmap /* CUtensorMap, host copy */, int64_t N,
                   int64_t T, const DevPolicy* pol_dev, const int32_t* cidx_dev, int32_t nc,
                   int32_t W, int32_t H, const DevPlatform& plat, int64_t nseg, int64_t seg_len,
-                  const SegRecords& rec, uint32_t* out_dec, int64_t dec_cstride, int* grid_out);
+                  const StreamWork& wk, int* grid_out);
 int stream_ctas_per_sm(int32_t W, int32_t H);
-
-// Resolves the segment carries of all C configs and writes the summaries.
-int launch_fixup(cudaStream_t s, int64_t N, int64_t T, int32_t C, const DevPlatform& plat,
-                 int64_t nseg, int64_t seg_len, const SegRecords& rec, magus_summary* out_summary,
-                 magus_base* out_base, uint32_t* out_dec);
 
 int launch_totals(cudaStream_t s, const magus_summary* summary, const magus_base* base, int64_t N,
                   int64_t T, int32_t C, uint64_t* totals);
