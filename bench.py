@@ -193,6 +193,7 @@ def run_ours(args):
     import torch.distributed as dist
 
     import paper_conf_sc_zhengspl25_b200 as magus
+    from paper_conf_sc_zhengspl25_b200 import dist as mdist
 
     world, rank, local = dist_env()
     if world != args.gpus:
@@ -215,7 +216,8 @@ def run_ours(args):
     C = len(pols)
     seed = SEED_BASE + args.config
     ctx = magus.Context(device=local, stream=stream)
-    x = ctx.gen_traces(seed, N, T, kind=kind, id0=rank * N)
+    id0, _ = mdist.shard(N * world, world, rank)     # weak scaling: N traces per GPU
+    x = ctx.gen_traces(seed, N, T, kind=kind, id0=id0)
     torch.cuda.synchronize()
 
     out = None
@@ -224,8 +226,7 @@ def run_ours(args):
         nonlocal out
         out = ctx.replay(x, pols, want_summary=False, want_base=False, want_decisions=want_dec,
                          want_totals=True, out=out)
-        if world > 1:
-            dist.all_reduce(out.totals, op=dist.ReduceOp.SUM)  # exact: integer words
+        mdist.allreduce_totals(out.totals)  # the one collective; exact (integer words)
         return ctx.sweep_best(out.totals)
 
     for _ in range(args.warmup):

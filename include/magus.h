@@ -234,6 +234,14 @@ magus_status magus_sweep_best(magus_ctx ctx, const uint64_t* totals,
                               int32_t n_params, int32_t* best,
                               magus_derived* best_row);
 
+/* Host-only forms (no context, no GPU): the same derivation and choice from
+ * host totals [n_params][MAGUS_TOT_WORDS] under *plat.  Used by the
+ * multi-rank glue after the all-reduce and by CPU tests. */
+magus_status magus_derive_host(const magus_platform* plat, const uint64_t* totals_host,
+                               magus_derived* out);
+magus_status magus_sweep_best_host(const magus_platform* plat, const uint64_t* totals_host,
+                                   int32_t n_params, int32_t* best, magus_derived* best_row);
+
 /* ---- synthetic traces (input generator; gen/magus_gen.h) --------------- */
 enum { MAGUS_GEN_MIX = 0, MAGUS_GEN_ADVERSARIAL = 1 };
 /* Writes traces id0 .. id0+n_traces-1 of the seeded Markov phase model to

@@ -103,18 +103,23 @@ _lib.magus_set_option.argtypes = [_vp, _i32, _i64]
 _lib.magus_policy_inspect.argtypes = [ctypes.POINTER(Policy), ctypes.POINTER(PolicyConsts)]
 _lib.magus_platform_inspect.argtypes = [ctypes.POINTER(Platform), ctypes.POINTER(PlatformConsts)]
 _lib.magus_get_stats.argtypes = [_vp, ctypes.POINTER(Stats)]
+_lib.magus_derive_host.argtypes = [ctypes.POINTER(Platform), _vp, ctypes.POINTER(Derived)]
+_lib.magus_sweep_best_host.argtypes = [ctypes.POINTER(Platform), _vp, _i32, ctypes.POINTER(_i32),
+                                       ctypes.POINTER(Derived)]
 _lib.magus_reset_stats.argtypes = [_vp]
 for _f in ("magus_init", "magus_destroy", "magus_set_stream", "magus_policy_preset", "magus_platform_preset",
            "magus_grid_sweep256", "magus_grid_fleet64", "magus_replay", "magus_replay_host",
            "magus_totals_derive", "magus_sweep_best", "magus_gen_traces", "magus_set_option",
-           "magus_get_stats", "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect"):
+           "magus_get_stats", "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
+           "magus_sweep_best_host"):
     getattr(_lib, _f).restype = ctypes.c_int
 
 EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_string", "magus_last_error",
             "magus_abi_version", "magus_policy_preset", "magus_platform_preset", "magus_grid_sweep256",
             "magus_grid_fleet64", "magus_replay", "magus_replay_host", "magus_totals_derive",
             "magus_sweep_best", "magus_gen_traces", "magus_set_option", "magus_get_stats",
-            "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect"]
+            "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
+            "magus_sweep_best_host"]
 
 
 class MagusError(RuntimeError):
@@ -170,6 +175,29 @@ def platform_inspect(p: Platform) -> dict:
     if st:
         raise MagusError(st, "platform_inspect")
     return {k: getattr(o, k) for k, _ in o._fields_}
+
+
+def derive_host(totals_row, platform: Platform | None = None) -> dict:
+    """Fleet fp64 quantities of one config from its integer totals (no GPU)."""
+    plat = platform if platform is not None else platform_preset()
+    w = np.ascontiguousarray(np.asarray(totals_row).view(np.uint64).reshape(TOT_WORDS))
+    d = Derived()
+    st = _lib.magus_derive_host(ctypes.byref(plat), _vp(w.ctypes.data), ctypes.byref(d))
+    if st:
+        raise MagusError(st, "derive_host")
+    return d.as_dict()
+
+
+def sweep_best_host(totals, platform: Platform | None = None) -> tuple[int, dict, bool]:
+    """(best, derived row, feasible) from host totals [C, 16] (no GPU)."""
+    plat = platform if platform is not None else platform_preset()
+    w = np.ascontiguousarray(np.asarray(totals).view(np.uint64).reshape(-1, TOT_WORDS))
+    best, d = _i32(), Derived()
+    st = _lib.magus_sweep_best_host(ctypes.byref(plat), _vp(w.ctypes.data), len(w), ctypes.byref(best),
+                                    ctypes.byref(d))
+    if st not in (OK, ERR_NO_FEASIBLE):
+        raise MagusError(st, "sweep_best_host")
+    return int(best.value), d.as_dict(), st == OK
 
 
 def make_policy(W=10, H=10, L=None, tau_inc=200.0, tau_dec=-500.0, t_hi=0.4) -> Policy:

@@ -38,6 +38,8 @@ struct magus_ctx_s {
   void* pol_host = nullptr;  // pinned staging
   size_t pol_host_bytes = 0;
   cudaEvent_t pol_copied = nullptr;
+  std::vector<uint64_t> best_host;   // sweep_best staging (size marker)
+  void* best_pinned = nullptr;
   std::vector<std::pair<std::pair<int, int>, std::vector<int32_t>>> groups;  // (W,H) -> configs
   std::vector<int64_t> group_offsets;                                        // into cidx
   // e2e staging (device)
@@ -398,6 +400,7 @@ magus_status magus_destroy(magus_ctx ctx) {
     if (ctx->scratch) cudaFree(ctx->scratch);
     if (ctx->pol_dev) cudaFree(ctx->pol_dev);
     if (ctx->pol_host) cudaFreeHost(ctx->pol_host);
+    if (ctx->best_pinned) cudaFreeHost(ctx->best_pinned);
     if (ctx->stage_dev) cudaFree(ctx->stage_dev);
     if (ctx->pol_copied) cudaEventDestroy(ctx->pol_copied);
     for (auto& pr : ctx->pending) {
@@ -619,16 +622,10 @@ magus_status magus_totals_derive(magus_ctx ctx, const uint64_t* totals_host, mag
   return MAGUS_OK;
 }
 
-magus_status magus_sweep_best(magus_ctx ctx, const uint64_t* totals, int32_t C, int32_t* best,
-                              magus_derived* best_row) {
-  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
-  if (!totals || C < 1 || !best) return fail(ctx, MAGUS_ERR_INVALID_ARG, "bad sweep_best arguments");
-  DeviceGuard dg(ctx->device);
-  std::vector<uint64_t> h((size_t)C * MAGUS_TOT_WORDS);
-  CK(cudaMemcpyAsync(h.data(), totals, h.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
-  CK(cudaStreamSynchronize(ctx->stream));
+static magus_status choose_best(const DevPlatform& dp, const uint64_t* h, int32_t C, int32_t* best,
+                                magus_derived* best_row) {
   std::vector<magus_derived> d((size_t)C);
-  for (int32_t c = 0; c < C; ++c) derive_totals(ctx->dplat, h.data() + (size_t)c * MAGUS_TOT_WORDS, &d[c]);
+  for (int32_t c = 0; c < C; ++c) derive_totals(dp, h + (size_t)c * MAGUS_TOT_WORDS, &d[c]);
   int32_t b = -1;
   for (int32_t c = 0; c < C; ++c)
     if (d[c].n_viol == 0 && (b < 0 || d[c].energy_j < d[b].energy_j)) b = c;
@@ -638,11 +635,45 @@ magus_status magus_sweep_best(magus_ctx ctx, const uint64_t* totals, int32_t C, 
     b = 0;
     for (int32_t c = 1; c < C; ++c)
       if (d[c].n_viol < d[b].n_viol || (d[c].n_viol == d[b].n_viol && d[c].energy_j < d[b].energy_j)) b = c;
-    ctx->err = "no config keeps every trace within the slowdown bound";
   }
   *best = b;
   if (best_row) *best_row = d[b];
   return st;
+}
+
+magus_status magus_sweep_best(magus_ctx ctx, const uint64_t* totals, int32_t C, int32_t* best,
+                              magus_derived* best_row) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  if (!totals || C < 1 || !best) return fail(ctx, MAGUS_ERR_INVALID_ARG, "bad sweep_best arguments");
+  DeviceGuard dg(ctx->device);
+  if (ctx->best_host.size() < (size_t)C * MAGUS_TOT_WORDS) {
+    if (ctx->best_pinned) cudaFreeHost(ctx->best_pinned);
+    ctx->best_pinned = nullptr;
+    CK(cudaMallocHost(&ctx->best_pinned, sizeof(uint64_t) * (size_t)C * MAGUS_TOT_WORDS));
+    ctx->best_host.resize((size_t)C * MAGUS_TOT_WORDS);
+  }
+  CK(cudaMemcpyAsync(ctx->best_pinned, totals, sizeof(uint64_t) * (size_t)C * MAGUS_TOT_WORDS,
+                     cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  magus_status st = choose_best(ctx->dplat, (const uint64_t*)ctx->best_pinned, C, best, best_row);
+  if (st == MAGUS_ERR_NO_FEASIBLE) ctx->err = "no config keeps every trace within the slowdown bound";
+  return st;
+}
+
+magus_status magus_derive_host(const magus_platform* plat, const uint64_t* totals_host,
+                               magus_derived* out) {
+  char msg[256];
+  if (!plat || !totals_host || !out || !validate_platform(*plat, msg, sizeof msg)) return MAGUS_ERR_INVALID_ARG;
+  derive_totals(make_dev_platform(*plat), totals_host, out);
+  return MAGUS_OK;
+}
+
+magus_status magus_sweep_best_host(const magus_platform* plat, const uint64_t* totals_host,
+                                   int32_t C, int32_t* best, magus_derived* best_row) {
+  char msg[256];
+  if (!plat || !totals_host || C < 1 || !best || !validate_platform(*plat, msg, sizeof msg))
+    return MAGUS_ERR_INVALID_ARG;
+  return choose_best(make_dev_platform(*plat), totals_host, C, best, best_row);
 }
 
 magus_status magus_gen_traces(magus_ctx ctx, uint64_t seed, int64_t id0, int64_t N, int64_t T,

@@ -31,10 +31,12 @@ __device__ __forceinline__ uint64_t q_literal(float x, double invB) {
 // Same quantity, strength-reduced (valid when x > xthr, i.e. RN(x*invB) > 1):
 // r24 = RN(x*invB*2^24) = RN(x*invB)*2^24 and RN(r24 - 2^24) = RN(r-1)*2^24
 // (power-of-two scaling commutes with round-to-nearest in the normal range).
+// s24 is in (0, 2^39], so floor(s24) = bits(RZ(s24 + 2^52)) - bits(2^52):
+// an fp64 add instead of the F2I conversion on the slow XU pipe.
 __device__ __forceinline__ uint64_t q_scaled(float x, double invB24) {
   double s24 = (double)x * invB24 - kQScale;
-  if (s24 > kQCapScaled) s24 = kQCapScaled;
-  return (uint64_t)s24;
+  s24 = fmin(s24, kQCapScaled);
+  return (uint64_t)__double_as_longlong(__dadd_rz(s24, 4503599627370496.0)) - 0x4330000000000000ULL;
 }
 
 // Model M finalisation of one (trace, config); fixed fp64
