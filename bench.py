@@ -216,6 +216,10 @@ def run_ours(args):
     C = len(pols)
     seed = SEED_BASE + args.config
     ctx = magus.Context(device=local, stream=stream)
+    if args.waves:
+        ctx.set_option(magus.OPT_WAVES, args.waves)
+    if args.segments:
+        ctx.set_option(magus.OPT_SEGMENTS, args.segments)
     id0, _ = mdist.shard(N * world, world, rank)     # weak scaling: N traces per GPU
     x = ctx.gen_traces(seed, N, T, kind=kind, id0=id0)
     torch.cuda.synchronize()
@@ -360,6 +364,8 @@ def main():
     ap.add_argument("--n-traces", type=int, default=0)
     ap.add_argument("--n-steps", type=int, default=0)
     ap.add_argument("--no-decisions", action="store_true")
+    ap.add_argument("--waves", type=int, default=0, help="MAGUS_OPT_WAVES (0 = library default)")
+    ap.add_argument("--segments", type=int, default=0, help="MAGUS_OPT_SEGMENTS (0 = auto)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -203,16 +203,19 @@ __device__ __forceinline__ uint32_t tail_mask(int64_t p0, int64_t T) {
   return (p0 + 32 <= T) ? ~0u : ((1u << (uint32_t)(T - p0)) - 1u);
 }
 
+#ifndef MAGUS_STAGES_REG
+#define MAGUS_STAGES_REG 3
+#endif
 template <int W_T>
 struct Stages {
   // register lag (compile-time W): a stage is free once its word is read;
   // runtime W reads the lag from the previous stage, held one word longer.
-  static constexpr int n = W_T > 0 ? 3 : 4;
+  static constexpr int n = W_T > 0 ? MAGUS_STAGES_REG : 4;
   static constexpr int smem = n * kStageFloats * 4;
 };
 
 template <int W_T, int H_T>
-__global__ void __launch_bounds__(kThreads, W_T > 0 ? 4 : 3)
+__global__ void __launch_bounds__(kThreads, W_T > 0 ? (MAGUS_STAGES_REG == 3 ? 4 : 3) : 3)
 stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
               const DevPolicy* __restrict__ pol, const int32_t* __restrict__ cidx, DevPlatform plat,
               int64_t nseg, int64_t seg_len, int32_t ngroups, int32_t nconf, StreamWork wk) {
@@ -221,6 +224,10 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
   __shared__ __align__(8) uint64_t full_bar[kStages];
   __shared__ __align__(8) uint64_t empty_bar[kStages];
   __shared__ uint32_t sh_ticket, sh_last, sh_last2;
+  // per-stage word constants, computed by the producer lane off the critical path
+  __shared__ unsigned long long st_mul[kStages];  // digest multiplier mix64(w) | 1
+  __shared__ uint32_t st_warm[kStages];           // positions t < W (no MDFS round yet)
+  __shared__ uint32_t st_tail[kStages];           // positions t < T
   __shared__ unsigned long long sh_red[kConsumerWarps][kTotAcc];
 
   if (threadIdx.x == 0) {
@@ -262,12 +269,18 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (warp == kConsumerWarps) {  // ---------------- producer warp ----------------
     if (lane == 0) {
+      int st = 0;
+      uint32_t ph = 0;
       for (int64_t j = 0; j < nwords; ++j) {
-        const int st = (int)(j % kStages);
-        if (j >= kStages) mbar_wait(&empty_bar[st], (uint32_t)((j / kStages) - 1) & 1u);
-        mbar_expect_tx(&full_bar[st], kStageBytes);
+        if (j >= kStages) mbar_wait(&empty_bar[st], ph ^ 1u);
+        const int64_t w = w_first + j, p0 = w * 32;
+        st_mul[st] = digest_mul(w);
+        st_warm[st] = (p0 >= W) ? 0u : ((W - p0) >= 32 ? ~0u : ((1u << (W - p0)) - 1u));
+        st_tail[st] = tail_mask(p0, T);
+        mbar_expect_tx(&full_bar[st], kStageBytes);  // arrive: releases the writes above
         tma_load_2d(sm + st * kStageFloats, &tmap, &full_bar[st], g * kTraces,
                     (int32_t)((w_first + j) * kRows));
+        if (++st == kStages) { st = 0; ph ^= 1u; }
       }
     }
     return;
@@ -289,13 +302,15 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
   uint32_t ev = 0, hi = 0, msr = 0, ch = 0, mdec = 0, mint = 0;
   unsigned long long qmin = 0, qmax = 0, qbase = 0, dig = 0, pqmin = 0, pqmax = 0, pdig = 0;
   uint32_t* dec_out = (wk.dec && valid) ? wk.dec + (int64_t)c * wk.dec_cstride + n : nullptr;
+  uint32_t* dec_ptr = dec_out ? dec_out + wt0 * N : nullptr;  // advances one word row per word
   double pd[W_T > 1 ? W_T - 1 : 1];  // previous word's last W-1 samples, widened
 #pragma unroll
   for (int k = 0; k < (W_T > 1 ? W_T - 1 : 1); ++k) pd[k] = 0.0;
 
+  int st = 0, pst = kStages - 1;
+  uint32_t ph = 0;
   for (int64_t j = 0; j < nwords; ++j) {
-    const int st = (int)(j % kStages);
-    mbar_wait(&full_bar[st], (uint32_t)(j / kStages) & 1u);
+    mbar_wait(&full_bar[st], ph);
     const float* cur = sm + st * kStageFloats + tid;
     const int64_t w = w_first + j;
     const int64_t p0 = w * 32;
@@ -319,7 +334,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
 #pragma unroll
       for (int k = 0; k < W_T - 1; ++k) pd[k] = xd[32 - (W_T - 1) + k];
     } else {
-      const float* prv = sm + ((j + kStages - 1) % kStages) * kStageFloats + tid;
+      const float* prv = sm + pst * kStageFloats + tid;
 #pragma unroll
       for (int i = 0; i < 32; ++i) {
         const float xi = cur[i * kTraces];
@@ -332,13 +347,13 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
         wmax = fmaxf(wmax, xi);
       }
     }
-    const uint32_t warm = (p0 >= W) ? 0u : ((W - p0) >= 32 ? ~0u : ((1u << (W - p0)) - 1u));
+    const uint32_t warm = st_warm[st];
     const uint32_t incv = incw & ~warm;          // p = +1
     const uint32_t decv = decw & ~warm & ~incv;  // p = -1 (line 4 before line 6)
     const uint32_t E = incv | decv;              // uncore_tune_ls.push_back(1)
 
     if (w >= wt0) {
-      const uint32_t outm = tail_mask(p0, T);
+      const uint32_t outm = st_tail[st];
       // Alg. 2 + override (l.9-15): hi_t from the H events before t
       const uint32_t HI = Window<H_T>::ge(E, Eprev, H, km) & ~warm;
       const uint32_t act = HI | E;                 // tune_uncore_freq calls
@@ -355,7 +370,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
       const uint32_t Dout = D & outm;
       mdec += __popc(Dout);
       mint += __popc(Lv & outm);
-      const uint64_t M = digest_mul(w);
+      const uint64_t M = st_mul[st];
       dig += (unsigned long long)Dout * M;
       uint32_t pre_int = 0;
       if (!seen) {  // prefix: decisions depend on the carry -> stored after the look-back
@@ -376,17 +391,24 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
           pre_dec = outm;
         }
         pdig += (unsigned long long)pre_dec * M;
-      } else if (dec_out) {
-        dec_out[w * N] = Dout;
+      } else if (dec_ptr) {
+        *dec_ptr = Dout;
       }
+      if (dec_ptr) dec_ptr += N;
       // model M stretch: sparse over the samples that need it
       uint32_t mq = smin & (Lv | pre_int) & outm;
-      while (mq) {  // order-free integer sums: scan from the top bit (one FLO)
-        const int i = 31 - __clz(mq);
-        mq ^= 1u << i;
-        const unsigned long long q = q_scaled(cur[i * kTraces], invB24_min);
-        if ((Lv >> i) & 1u) qmin += q;
-        if ((pre_int >> i) & 1u) pqmin += q;
+      while (mq) {  // order-free integer sums; two independent chains per trip
+        const int i1 = 31 - __clz(mq);
+        mq ^= 1u << i1;
+        const int i2 = mq ? 31 - __clz(mq) : i1;
+        const uint32_t m2 = mq ? 1u << i2 : 0u;
+        mq ^= m2;
+        const unsigned long long q1 = q_scaled(cur[i1 * kTraces], invB24_min);
+        const unsigned long long q2 = m2 ? q_scaled(cur[i2 * kTraces], invB24_min) : 0ULL;
+        if ((Lv >> i1) & 1u) qmin += q1;
+        if ((pre_int >> i1) & 1u) pqmin += q1;
+        if (Lv & m2) qmin += q2;
+        if (pre_int & m2) pqmin += q2;
       }
       if (wmax > xthr_max) {  // some sample exceeds even the capacity at max
         uint32_t mx = smin & outm;  // x > xthr_max implies x > xthr_min
@@ -410,8 +432,10 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
     if constexpr (W_T > 0) {
       if (lane == 0) mbar_arrive(&empty_bar[st]);                      // word read: free
     } else {
-      if (j >= 1 && lane == 0) mbar_arrive(&empty_bar[(j - 1) % kStages]);  // lag read: free
+      if (j >= 1 && lane == 0) mbar_arrive(&empty_bar[pst]);           // lag read: free
     }
+    pst = st;
+    if (++st == kStages) { st = 0; ph ^= 1u; }
   }
 
   // ---------------- epilogue: publish, look back, correct ----------------
