@@ -220,6 +220,8 @@ def run_ours(args):
         ctx.set_option(magus.OPT_WAVES, args.waves)
     if args.segments:
         ctx.set_option(magus.OPT_SEGMENTS, args.segments)
+    if args.bundle:
+        ctx.set_option(magus.OPT_BUNDLE, args.bundle)
     id0, _ = mdist.shard(N * world, world, rank)     # weak scaling: N traces per GPU
     x = ctx.gen_traces(seed, N, T, kind=kind, id0=id0)
     torch.cuda.synchronize()
@@ -366,6 +368,7 @@ def main():
     ap.add_argument("--no-decisions", action="store_true")
     ap.add_argument("--waves", type=int, default=0, help="MAGUS_OPT_WAVES (0 = library default)")
     ap.add_argument("--segments", type=int, default=0, help="MAGUS_OPT_SEGMENTS (0 = auto)")
+    ap.add_argument("--bundle", type=int, default=0, help="MAGUS_OPT_BUNDLE (0 = auto, 1, 2, 4)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-cpu-baseline", action="store_true")

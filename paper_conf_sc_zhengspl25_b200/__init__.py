@@ -24,7 +24,7 @@ OK, ERR_INVALID_ARG, ERR_NOT_INITIALIZED, ERR_CUDA, ERR_NCCL, ERR_OOM, ERR_UNSUP
 POLICY_PAPER_DEFAULT, POLICY_PAPER_PARETO = 0, 1
 PLATFORM_INTEL_A100, PLATFORM_INTEL_MAX1550 = 0, 1
 GEN_MIX, GEN_ADVERSARIAL = 0, 1
-OPT_KERNEL, OPT_SEGMENTS, OPT_TIMING, OPT_WAVES = 0, 1, 2, 3
+OPT_KERNEL, OPT_SEGMENTS, OPT_TIMING, OPT_WAVES, OPT_BUNDLE = 0, 1, 2, 3, 4
 KERNEL_AUTO, KERNEL_REFERENCE, KERNEL_STREAM = 0, 1, 2
 TOT_WORDS = 16
 TOT_NAMES = ["n_traces", "n_viol", "events", "hi_rounds", "msr_writes", "changes", "min_dec",

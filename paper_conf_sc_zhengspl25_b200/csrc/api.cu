@@ -40,8 +40,14 @@ struct magus_ctx_s {
   cudaEvent_t pol_copied = nullptr;
   std::vector<uint64_t> best_host;   // sweep_best staging (size marker)
   void* best_pinned = nullptr;
-  std::vector<std::pair<std::pair<int, int>, std::vector<int32_t>>> groups;  // (W,H) -> configs
-  std::vector<int64_t> group_offsets;                                        // into cidx
+  struct LaunchGroup {
+    int32_t W, H, NB;   // kernel specialisation
+    int64_t off;        // first bundle (rows of NB config indices) in the device table
+    int32_t nbund;
+  };
+  std::vector<LaunchGroup> groups;  // one stream launch each
+  int64_t opt_bundle = 0;           // 0 auto, else force NB in {1, 2, 4}
+  int64_t uploaded_bundle_opt = -1;
   // e2e staging (device)
   void* stage_dev = nullptr;
   size_t stage_bytes = 0;
@@ -127,22 +133,42 @@ bool same_params(const std::vector<magus_policy>& a, const magus_policy* b, int3
   return std::memcmp(a.data(), b, sizeof(magus_policy) * (size_t)n) == 0;
 }
 
-// Uploads DevPolicy[C] + config index lists of the (W,H) groups.
+// Uploads DevPolicy[C] and the bundle table.  Configs are grouped by (W, H)
+// (one kernel specialisation per group), and inside a group into bundles of
+// NB configs with bit-identical inverted Alg. 1 thresholds (same L, tau_inc,
+// tau_dec up to rounding): a bundle shares Delta, the event word and the Alg. 2
+// window count, and differs only in k (t_hi).
 magus_status upload_policies(magus_ctx ctx, const magus_policy* params, int32_t C) {
-  if (same_params(ctx->last_params, params, C) && ctx->pol_dev) return MAGUS_OK;
+  if (same_params(ctx->last_params, params, C) && ctx->pol_dev &&
+      ctx->uploaded_bundle_opt == ctx->opt_bundle)
+    return MAGUS_OK;
   std::vector<DevPolicy> dp((size_t)C);
-  std::map<std::pair<int, int>, std::vector<int32_t>> g;
+  std::map<std::pair<int, int>, std::map<std::pair<uint64_t, uint64_t>, std::vector<int32_t>>> g;
   for (int32_t c = 0; c < C; ++c) {
     dp[c] = make_dev_policy(params[c]);
-    g[{params[c].window, params[c].history}].push_back(c);
+    uint64_t ki, kd;
+    std::memcpy(&ki, &dp[c].d_inc, 8);
+    std::memcpy(&kd, &dp[c].d_dec, 8);
+    g[{params[c].window, params[c].history}][{ki, kd}].push_back(c);
   }
-  ctx->groups.assign(g.begin(), g.end());
-  ctx->group_offsets.clear();
-  std::vector<int32_t> cidx;
-  for (auto& kv : ctx->groups) {
-    ctx->group_offsets.push_back((int64_t)cidx.size());
-    cidx.insert(cidx.end(), kv.second.begin(), kv.second.end());
+  ctx->groups.clear();
+  std::vector<int32_t> table;
+  for (auto& wh : g) {
+    size_t maxsz = 1;
+    for (auto& b : wh.second) maxsz = std::max(maxsz, b.second.size());
+    int32_t NB = ctx->opt_bundle ? (int32_t)ctx->opt_bundle : (maxsz >= 3 ? 4 : (int32_t)maxsz);
+    magus_ctx_s::LaunchGroup lg{wh.first.first, wh.first.second, NB, 0, 0};
+    lg.off = (int64_t)table.size();
+    for (auto& b : wh.second) {
+      const auto& v = b.second;
+      for (size_t i = 0; i < v.size(); i += (size_t)NB) {
+        for (int32_t k = 0; k < NB; ++k) table.push_back(i + k < v.size() ? v[i + k] : -1);
+        lg.nbund++;
+      }
+    }
+    ctx->groups.push_back(lg);
   }
+  std::vector<int32_t>& cidx = table;
   const size_t pol_bytes = align_up(sizeof(DevPolicy) * (size_t)C, 256);
   const size_t need = pol_bytes + sizeof(int32_t) * cidx.size();
   if (ctx->pol_copied) CK(cudaEventSynchronize(ctx->pol_copied));  // pinned buffer reuse
@@ -165,6 +191,7 @@ magus_status upload_policies(magus_ctx ctx, const magus_policy* params, int32_t 
   if (!ctx->pol_copied) CK(cudaEventCreateWithFlags(&ctx->pol_copied, cudaEventDisableTiming));
   CK(cudaEventRecord(ctx->pol_copied, ctx->stream));
   ctx->last_params.assign(params, params + C);
+  ctx->uploaded_bundle_opt = ctx->opt_bundle;
   return MAGUS_OK;
 }
 
@@ -174,11 +201,11 @@ const int32_t* dev_cidx(magus_ctx ctx, int64_t off) {
   return (const int32_t*)((const char*)ctx->pol_dev + pol_bytes) + off;
 }
 
-int ctas_per_sm(magus_ctx ctx, int W, int H) {
-  auto key = std::make_pair(W, H);
+int ctas_per_sm(magus_ctx ctx, int W, int H, int NB) {
+  auto key = std::make_pair(W * 8 + NB, H);
   auto it = ctx->ctas_cache.find(key);
   if (it != ctx->ctas_cache.end()) return it->second;
-  int v = stream_ctas_per_sm(W, H);
+  int v = stream_ctas_per_sm(W, H, NB);
   ctx->ctas_cache[key] = v;
   return v;
 }
@@ -433,6 +460,11 @@ magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value) {
     case MAGUS_OPT_TIMING:
       ctx->opt_timing = value ? 1 : 0;
       return MAGUS_OK;
+    case MAGUS_OPT_BUNDLE:
+      if (value != 0 && value != 1 && value != 2 && value != 4)
+        return fail(ctx, MAGUS_ERR_INVALID_ARG, "bundle option must be 0, 1, 2 or 4");
+      ctx->opt_bundle = value;
+      return MAGUS_OK;
     case MAGUS_OPT_WAVES:
       if (value < 1 || value > 64) return fail(ctx, MAGUS_ERR_INVALID_ARG, "waves not in [1, 64]");
       ctx->opt_waves = value;
@@ -472,12 +504,19 @@ magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t N, int64_t
       nseg = ctx->opt_segments;
     } else {
       int per_sm = 1 << 30;
-      for (auto& g : ctx->groups) per_sm = std::min(per_sm, ctas_per_sm(ctx, g.first.first, g.first.second));
+      int64_t nbund = 0;
+      for (auto& g : ctx->groups) {
+        per_sm = std::min(per_sm, ctas_per_sm(ctx, g.W, g.H, g.NB));
+        nbund += g.nbund;
+      }
       if (per_sm < 1) per_sm = 1;
       const int64_t slots = (int64_t)ctx->sms * per_sm * ctx->opt_waves;
-      nseg = std::max<int64_t>(1, (slots + ngroups * C - 1) / (ngroups * C));
+      nseg = std::max<int64_t>(1, (slots + ngroups * nbund - 1) / (ngroups * nbund));
     }
     seg_len = ((T + nseg - 1) / nseg + 31) / 32 * 32;
+    bool packed = false;  // NB > 1 packs per-segment counters in 16 bits
+    for (auto& g : ctx->groups) packed = packed || g.NB > 1;
+    if (packed && seg_len > 65504) seg_len = 65504;
     const int64_t min_len = 512;  // keeps the halo re-read below ~6 %
     if (ctx->opt_segments == 0 && seg_len < min_len) seg_len = std::min<int64_t>(min_len, ((T + 31) / 32) * 32);
     nseg = (T + seg_len - 1) / seg_len;
@@ -556,9 +595,8 @@ magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t N, int64_t
     for (size_t gi = 0; gi < ctx->groups.size(); ++gi) {
       auto& g = ctx->groups[gi];
       int grid = 0;
-      int r = launch_stream(ctx->stream, &map, N, T, dev_policies(ctx), dev_cidx(ctx, ctx->group_offsets[gi]),
-                            (int32_t)g.second.size(), g.first.first, g.first.second, ctx->dplat, nseg,
-                            seg_len, wk, &grid);
+      int r = launch_stream(ctx->stream, &map, N, T, dev_policies(ctx), dev_cidx(ctx, g.off), g.nbund,
+                            g.NB, g.W, g.H, ctx->dplat, nseg, seg_len, wk, &grid);
       if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "stream kernel launch");
       launched += r;
       grid_total += grid;

@@ -118,10 +118,14 @@ __device__ __forceinline__ void fa(uint32_t a, uint32_t b, uint32_t c, uint32_t&
   s = a ^ b ^ c;
   cy = (a & b) | (c & (a ^ b));
 }
+// Bit-sliced count of the H events before each of the 32 positions
+// (positions < 0 come from the previous word Ep): c[0..NBITS) per position.
 template <int H>
-struct Window {  // compile-time H: ripple-carry bit-sliced counter (6 bits, H <= 32)
-  static __device__ __forceinline__ uint32_t ge(uint32_t E, uint32_t Ep, int, const KMask& km) {
-    uint32_t c[6] = {0, 0, 0, 0, 0, 0};
+struct Window {  // compile-time H <= 32: ripple-carry counter, 6 bits
+  static constexpr int NBITS = 6;
+  static __device__ __forceinline__ void count(uint32_t E, uint32_t Ep, int, uint32_t* c) {
+#pragma unroll
+    for (int l = 0; l < 6; ++l) c[l] = 0;
 #pragma unroll
     for (int j = 1; j <= H; ++j) {
       uint32_t b = __funnelshift_lc(Ep, E, j);  // clamps: j = 32 -> Ep
@@ -132,12 +136,12 @@ struct Window {  // compile-time H: ripple-carry bit-sliced counter (6 bits, H <
         b = t;
       }
     }
-    return ge_k<6>(c, km);
   }
 };
 template <>
 struct Window<10> {  // the paper's H = 10 (P@24182): carry-save tree, 16 LOP3
-  static __device__ __forceinline__ uint32_t ge(uint32_t E, uint32_t Ep, int, const KMask& km) {
+  static constexpr int NBITS = 4;
+  static __device__ __forceinline__ void count(uint32_t E, uint32_t Ep, int, uint32_t* c) {
     uint32_t s[10];
 #pragma unroll
     for (int j = 0; j < 10; ++j) s[j] = __funnelshift_l(Ep, E, j + 1);
@@ -146,20 +150,20 @@ struct Window<10> {  // the paper's H = 10 (P@24182): carry-save tree, 16 LOP3
     fa(s[3], s[4], s[5], b0, b1);
     fa(s[6], s[7], s[8], c0, c1);
     fa(a0, b0, c0, d0, d1);
-    uint32_t c[4];
     c[0] = d0 ^ s[9];
     const uint32_t e1 = d0 & s[9];
     fa(a1, b1, c1, f1, f2);
     fa(d1, e1, f1, c[1], g2);
     c[2] = f2 ^ g2;
     c[3] = f2 & g2;
-    return ge_k<4>(c, km);
   }
 };
 template <>
 struct Window<0> {  // runtime H <= 32
-  static __device__ __forceinline__ uint32_t ge(uint32_t E, uint32_t Ep, int H, const KMask& km) {
-    uint32_t c[6] = {0, 0, 0, 0, 0, 0};
+  static constexpr int NBITS = 6;
+  static __device__ __forceinline__ void count(uint32_t E, uint32_t Ep, int H, uint32_t* c) {
+#pragma unroll
+    for (int l = 0; l < 6; ++l) c[l] = 0;
     for (int j = 1; j <= H; ++j) {
       uint32_t b = __funnelshift_lc(Ep, E, j);  // clamps: j = 32 -> Ep
 #pragma unroll
@@ -169,7 +173,6 @@ struct Window<0> {  // runtime H <= 32
         b = t;
       }
     }
-    return ge_k<6>(c, km);
   }
 };
 
@@ -203,23 +206,48 @@ __device__ __forceinline__ uint32_t tail_mask(int64_t p0, int64_t T) {
   return (p0 + 32 <= T) ? ~0u : ((1u << (uint32_t)(T - p0)) - 1u);
 }
 
-#ifndef MAGUS_STAGES_REG
-#define MAGUS_STAGES_REG 3
-#endif
 template <int W_T>
 struct Stages {
   // register lag (compile-time W): a stage is free once its word is read;
   // runtime W reads the lag from the previous stage, held one word longer.
-  static constexpr int n = W_T > 0 ? MAGUS_STAGES_REG : 4;
+  static constexpr int n = W_T > 0 ? 3 : 4;
   static constexpr int smem = n * kStageFloats * 4;
 };
+// CTAs per SM the launch bounds aim for: NB configs per thread cost registers
+template <int W_T, int NB>
+struct Occ {
+  static constexpr int v = NB == 1 ? (W_T > 0 ? 4 : 3) : 3;
+};
 
-template <int W_T, int H_T>
-__global__ void __launch_bounds__(kThreads, W_T > 0 ? (MAGUS_STAGES_REG == 3 ? 4 : 3) : 3)
+// Per-config state of a bundle (NB configs that share W, H, L, tau_inc and
+// tau_dec and differ only in t_hi, i.e. in k).  Hot state lives in registers
+// (arrays indexed by compile-time constants only); state touched once per
+// segment or only on rare paths lives in shared memory, [k][thread].
+// For NB > 1 the per-segment counters are packed in 16-bit pairs (the host
+// keeps segments <= 65,504 steps), which keeps NB = 4 at 3 CTAs/SM.
+template <int NB>
+struct BundleRegs {
+  uint32_t cnt_a[NB];  // NB == 1: hi;   NB > 1: hi | msr << 16
+  uint32_t cnt_b[NB];  // NB == 1: msr;  NB > 1: mdec | mint << 16
+  uint32_t cnt_c[NB];  // NB == 1: mdec; NB > 1: ch
+  uint32_t cnt_d[NB];  // NB == 1: mint, ch packed separately below
+  uint32_t cnt_e[NB];
+  unsigned long long qmin[NB], dig[NB], pqmin[NB];
+  uint32_t carry, seen, va, last;  // bit k per config
+};
+struct BundleSmem {  // rarely touched, per (config slot, thread)
+  unsigned long long qmax, pqmax, pdig;
+  int32_t apos, wa;
+  uint32_t dwa, pre_dec_a;
+};
+
+template <int W_T, int H_T, int NB>
+__global__ void __launch_bounds__(kThreads, Occ<W_T, NB>::v)
 stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
-              const DevPolicy* __restrict__ pol, const int32_t* __restrict__ cidx, DevPlatform plat,
-              int64_t nseg, int64_t seg_len, int32_t ngroups, int32_t nconf, StreamWork wk) {
+              const DevPolicy* __restrict__ pol, const int32_t* __restrict__ bundles, DevPlatform plat,
+              int64_t nseg, int64_t seg_len, int32_t ngroups, int32_t nbund, StreamWork wk) {
   constexpr int kStages = Stages<W_T>::n;
+  constexpr bool kPack = NB > 1;
   extern __shared__ __align__(1024) float sm[];
   __shared__ __align__(8) uint64_t full_bar[kStages];
   __shared__ __align__(8) uint64_t empty_bar[kStages];
@@ -229,6 +257,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
   __shared__ uint32_t st_warm[kStages];           // positions t < W (no MDFS round yet)
   __shared__ uint32_t st_tail[kStages];           // positions t < T
   __shared__ unsigned long long sh_red[kConsumerWarps][kTotAcc];
+  __shared__ BundleSmem bs[NB][kTraces];
 
   if (threadIdx.x == 0) {
     sh_ticket = atomicAdd(wk.ticket, 1u);  // launch-order work ticket
@@ -238,22 +267,27 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  // zero the ring (the runtime-W path's first word reads a "previous" stage)
-  for (int i = threadIdx.x; i < kStages * kStageFloats; i += kThreads) sm[i] = 0.0f;
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  if constexpr (W_T == 0) {  // the runtime-W path's first word reads a "previous" stage
+    for (int i = threadIdx.x; i < kStages * kStageFloats; i += kThreads) sm[i] = 0.0f;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
   __syncthreads();
 
-  // ticket -> (segment, config, group), segment-major so that the predecessor
-  // segment of the same (config, group) always holds a smaller ticket
+  // ticket -> (segment, bundle, group), segment-major so that the predecessor
+  // segment of the same (bundle, group) always holds a smaller ticket
   const uint32_t ticket = sh_ticket;
-  const int64_t per_seg = (int64_t)ngroups * nconf;
+  const int64_t per_seg = (int64_t)ngroups * nbund;
   const int64_t s = ticket / per_seg;
   const int32_t rem = (int32_t)(ticket - s * per_seg);
-  const int32_t c = cidx[rem / ngroups];  // global config index
+  const int32_t bidx = rem / ngroups;
   const int32_t g = rem % ngroups;
+  int32_t cfg[NB];
+#pragma unroll
+  for (int k = 0; k < NB; ++k) cfg[k] = bundles[bidx * NB + k];  // global config, -1 = pad
+  const int32_t c0 = cfg[0];
   const int64_t t0 = s * seg_len;
   const int64_t t1 = (t0 + seg_len < T) ? t0 + seg_len : T;
-  const DevPolicy P = pol[c];
+  const DevPolicy P = pol[c0];
   const int W = W_T > 0 ? W_T : P.W;
   const int H = H_T > 0 ? H_T : P.H;
   const int64_t wt0 = t0 >> 5;
@@ -286,23 +320,32 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
     return;
   }
 
-  // ---------------- consumer: one trace per thread ----------------
+  // ---------------- consumer: one trace x NB configs per thread ----------------
   const int tid = threadIdx.x;
   const int64_t n = (int64_t)g * kTraces + tid;
   const bool valid = n < N;
-  const double d_inc = P.d_inc, d_dec = P.d_dec;
-  const KMask km = make_kmask(P.k);
+  const double d_inc = P.d_inc, d_dec = P.d_dec;  // shared by the bundle
+  int32_t kk[NB];
+#pragma unroll
+  for (int k = 0; k < NB; ++k) kk[k] = cfg[k] >= 0 ? pol[cfg[k]].k : 0x3F;
   const float xthr_min = plat.xthr_min, xthr_max = plat.xthr_max;
   const double invB24_min = plat.invB24_min, invB24_max = plat.invB24_max;
   const uint32_t hyp = (s > 0) ? 1u : 0u;  // segment 0 starts from the true dec[-1] = max
-  uint32_t Eprev = 0, carry = hyp, Dlast = 0;
-  bool seen = false;
-  uint32_t Va = 0, Dwa = 0, pre_dec_a = 0;
-  int64_t apos = -1, wa = -1;
-  uint32_t ev = 0, hi = 0, msr = 0, ch = 0, mdec = 0, mint = 0;
-  unsigned long long qmin = 0, qmax = 0, qbase = 0, dig = 0, pqmin = 0, pqmax = 0, pdig = 0;
-  uint32_t* dec_out = (wk.dec && valid) ? wk.dec + (int64_t)c * wk.dec_cstride + n : nullptr;
-  uint32_t* dec_ptr = dec_out ? dec_out + wt0 * N : nullptr;  // advances one word row per word
+  const uint32_t last_bit = (uint32_t)((t1 - 1) & 31);
+  BundleRegs<NB> B;
+#pragma unroll
+  for (int k = 0; k < NB; ++k) {
+    B.cnt_a[k] = 0; B.cnt_b[k] = 0; B.cnt_c[k] = 0; B.cnt_d[k] = 0; B.cnt_e[k] = 0;
+    B.qmin[k] = 0; B.dig[k] = 0; B.pqmin[k] = 0;
+    bs[k][tid].qmax = 0; bs[k][tid].pqmax = 0; bs[k][tid].pdig = 0;
+    bs[k][tid].apos = -1; bs[k][tid].wa = -1; bs[k][tid].dwa = 0; bs[k][tid].pre_dec_a = 0;
+  }
+  B.carry = hyp ? (1u << NB) - 1u : 0u;
+  B.seen = 0; B.va = 0; B.last = 0;
+  uint32_t Eprev = 0, ev = 0;
+  unsigned long long qbase = 0;
+  const bool want_dec = wk.dec != nullptr && valid;
+  uint32_t* dec_row = want_dec ? wk.dec + wt0 * N + n : nullptr;  // + c * dec_cstride
   double pd[W_T > 1 ? W_T - 1 : 1];  // previous word's last W-1 samples, widened
 #pragma unroll
   for (int k = 0; k < (W_T > 1 ? W_T - 1 : 1); ++k) pd[k] = 0.0;
@@ -354,78 +397,102 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
 
     if (w >= wt0) {
       const uint32_t outm = st_tail[st];
-      // Alg. 2 + override (l.9-15): hi_t from the H events before t
-      const uint32_t HI = Window<H_T>::ge(E, Eprev, H, km) & ~warm;
-      const uint32_t act = HI | E;                 // tune_uncore_freq calls
-      const uint32_t A = act | warm;               // positions that set the frequency
-      const uint32_t V = decv & ~HI;               // ... to min (l.25)
-      const uint32_t D = forward_fill(A, V, carry ? ~0u : 0u);
-      const uint32_t Lv = (D << 1) | carry;        // interval level = dec[t-1]
-      ev += __popc(E & outm);
-      hi += __popc(HI & outm);
-      msr += __popc(act & outm);
-      uint32_t chm = (D ^ Lv) & outm;
-      if (p0 == 0) chm &= ~1u;
-      ch += __popc(chm);
-      const uint32_t Dout = D & outm;
-      mdec += __popc(Dout);
-      mint += __popc(Lv & outm);
       const uint64_t M = st_mul[st];
-      dig += (unsigned long long)Dout * M;
-      uint32_t pre_int = 0;
-      if (!seen) {  // prefix: decisions depend on the carry -> stored after the look-back
-        const uint32_t Am = A & outm;
-        uint32_t pre_dec;
-        if (Am) {
-          const int i = __ffs(Am) - 1;
-          seen = true;
-          apos = p0 + i;
-          Va = (V >> i) & 1u;
-          pre_int = (i == 31) ? ~0u : ((2u << i) - 1u);
-          pre_dec = (1u << i) - 1u;
-          wa = w;
-          Dwa = Dout;
-          pre_dec_a = pre_dec;
+      const bool final_word = (w == wend - 1);
+      ev += __popc(E & outm);
+      // Alg. 2 (l.9): the count of the H previous events, shared by the bundle
+      uint32_t cnt[Window<H_T>::NBITS];
+      Window<H_T>::count(E, Eprev, H, cnt);
+      uint32_t Lv[NB], pre_int[NB];
+      uint32_t need_q = 0;
+#pragma unroll
+      for (int k = 0; k < NB; ++k) {
+        const uint32_t ck = (B.carry >> k) & 1u;
+        const uint32_t HI = ge_k<Window<H_T>::NBITS>(cnt, make_kmask(kk[k])) & ~warm;
+        const uint32_t act = HI | E;                 // tune_uncore_freq calls (l.11/19/25)
+        const uint32_t A = act | warm;               // positions that set the frequency
+        const uint32_t V = decv & ~HI;               // ... to min (l.25)
+        const uint32_t D = forward_fill(A, V, ck ? ~0u : 0u);
+        Lv[k] = (D << 1) | ck;                       // interval level = dec[t-1]
+        uint32_t chm = (D ^ Lv[k]) & outm;
+        if (p0 == 0) chm &= ~1u;
+        const uint32_t Dout = D & outm;
+        if constexpr (kPack) {
+          B.cnt_a[k] += (uint32_t)__popc(HI & outm) | ((uint32_t)__popc(act & outm) << 16);
+          B.cnt_b[k] += (uint32_t)__popc(Dout) | ((uint32_t)__popc(Lv[k] & outm) << 16);
+          B.cnt_c[k] += (uint32_t)__popc(chm);
         } else {
-          pre_int = outm;
-          pre_dec = outm;
+          B.cnt_a[k] += __popc(HI & outm);
+          B.cnt_b[k] += __popc(act & outm);
+          B.cnt_c[k] += __popc(Dout);
+          B.cnt_d[k] += __popc(Lv[k] & outm);
+          B.cnt_e[k] += __popc(chm);
         }
-        pdig += (unsigned long long)pre_dec * M;
-      } else if (dec_ptr) {
-        *dec_ptr = Dout;
+        B.dig[k] += (unsigned long long)Dout * M;
+        pre_int[k] = 0;
+        if (!((B.seen >> k) & 1u)) {  // prefix: depends on the carry -> resolved later
+          const uint32_t Am = A & outm;
+          uint32_t pre_dec;
+          if (Am) {
+            const int i = __ffs(Am) - 1;
+            B.seen |= 1u << k;
+            B.va |= ((V >> i) & 1u) << k;
+            pre_int[k] = (i == 31) ? ~0u : ((2u << i) - 1u);
+            pre_dec = (1u << i) - 1u;
+            bs[k][tid].apos = (int32_t)(p0 + i - t0);
+            bs[k][tid].wa = (int32_t)(w - wt0);
+            bs[k][tid].dwa = Dout;
+            bs[k][tid].pre_dec_a = pre_dec;
+          } else {
+            pre_int[k] = outm;
+            pre_dec = outm;
+          }
+          bs[k][tid].pdig += (unsigned long long)pre_dec * M;
+        } else if (want_dec && cfg[k] >= 0) {
+          dec_row[(int64_t)cfg[k] * wk.dec_cstride] = Dout;
+        }
+        need_q |= (Lv[k] | pre_int[k]);
+        B.carry = (B.carry & ~(1u << k)) | ((D >> 31) << k);
+        if (final_word) B.last |= ((D >> last_bit) & 1u) << k;
       }
-      if (dec_ptr) dec_ptr += N;
-      // model M stretch: sparse over the samples that need it
-      uint32_t mq = smin & (Lv | pre_int) & outm;
+      if (dec_row) dec_row += N;
+      // model M stretch at min: once per sample, shared by the bundle
+      uint32_t mq = smin & need_q & outm;
       while (mq) {  // order-free integer sums; two independent chains per trip
         const int i1 = 31 - __clz(mq);
-        mq ^= 1u << i1;
+        const uint32_t m1 = 1u << i1;
+        mq ^= m1;
         const int i2 = mq ? 31 - __clz(mq) : i1;
         const uint32_t m2 = mq ? 1u << i2 : 0u;
         mq ^= m2;
         const unsigned long long q1 = q_scaled(cur[i1 * kTraces], invB24_min);
         const unsigned long long q2 = m2 ? q_scaled(cur[i2 * kTraces], invB24_min) : 0ULL;
-        if ((Lv >> i1) & 1u) qmin += q1;
-        if ((pre_int >> i1) & 1u) pqmin += q1;
-        if (Lv & m2) qmin += q2;
-        if (pre_int & m2) pqmin += q2;
+#pragma unroll
+        for (int k = 0; k < NB; ++k) {
+          if (Lv[k] & m1) B.qmin[k] += q1;
+          if (pre_int[k] & m1) B.pqmin[k] += q1;
+          if (Lv[k] & m2) B.qmin[k] += q2;
+          if (pre_int[k] & m2) B.pqmin[k] += q2;
+        }
       }
-      if (wmax > xthr_max) {  // some sample exceeds even the capacity at max
+      if (wmax > xthr_max) {  // some sample exceeds even the capacity at max (rare)
         uint32_t mx = smin & outm;  // x > xthr_max implies x > xthr_min
         while (mx) {
           const int i = 31 - __clz(mx);
-          mx ^= 1u << i;
+          const uint32_t m1 = 1u << i;
+          mx ^= m1;
           const float xi = cur[i * kTraces];
           if (xi > xthr_max) {
             const unsigned long long q = q_scaled(xi, invB24_max);
             qbase += q;
-            if (!((Lv >> i) & 1u)) qmax += q;
-            if ((pre_int >> i) & 1u) pqmax += q;
+#pragma unroll
+            for (int k = 0; k < NB; ++k) {
+              if (!(Lv[k] & m1)) bs[k][tid].qmax += q;
+              if (pre_int[k] & m1) bs[k][tid].pqmax += q;
+            }
           }
         }
       }
-      carry = D >> 31;
-      Dlast = D;
     }
     Eprev = E;
     __syncwarp();
@@ -439,44 +506,66 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
   }
 
   // ---------------- epilogue: publish, look back, correct ----------------
-  const uint32_t last_min = (Dlast >> (uint32_t)((t1 - 1) & 31)) & 1u;
-  uint32_t* status = wk.status + ((int64_t)c * nseg) * N + n;
-  if (valid) st_release(status + s * N, (wk.epoch << 3) | 1u | (seen ? 2u : 0u) | (last_min << 2));
-  uint32_t cin = 0;  // true dec[t0-1]
-  if (valid && s > 0) {
-    for (int64_t jj = s - 1; jj >= 0; --jj) {
-      uint32_t v;
-      while (((v = ld_acquire(status + jj * N)) >> 3) != wk.epoch) __nanosleep(32);
-      if (v & 2u) { cin = (v >> 2) & 1u; break; }
-    }
+#pragma unroll
+  for (int k = 0; k < NB; ++k) {
+    const int32_t c = cfg[k];
+    if (!valid || c < 0) continue;
+    const uint32_t seen = (B.seen >> k) & 1u, last_min = (B.last >> k) & 1u;
+    uint32_t* status = wk.status + ((int64_t)c * nseg) * N + n;
+    st_release(status + s * N, (wk.epoch << 3) | 1u | (seen << 1) | (last_min << 2));
   }
-  if (valid) {
-    if (cin != hyp) {
-      const int64_t n_int = seen ? apos - t0 + 1 : t1 - t0;
-      const int64_t n_dec = seen ? apos - t0 : t1 - t0;
-      if (hyp) {  // assumed min, truly max
-        mint -= (uint32_t)n_int; mdec -= (uint32_t)n_dec;
-        qmin -= pqmin; qmax += pqmax; dig -= pdig;
-      } else {    // assumed max, truly min
-        mint += (uint32_t)n_int; mdec += (uint32_t)n_dec;
-        qmin += pqmin; qmax -= pqmax; dig += pdig;
+#pragma unroll
+  for (int k = 0; k < NB; ++k) {
+    const int32_t c = cfg[k];
+    if (!valid || c < 0) continue;
+    const bool seen = (B.seen >> k) & 1u;
+    const BundleSmem& S = bs[k][tid];
+    uint32_t* status = wk.status + ((int64_t)c * nseg) * N + n;
+    uint32_t cin = 0;  // true dec[t0-1]
+    if (s > 0) {
+      for (int64_t jj = s - 1; jj >= 0; --jj) {
+        uint32_t v;
+        while (((v = ld_acquire(status + jj * N)) >> 3) != wk.epoch) __nanosleep(32);
+        if (v & 2u) { cin = (v >> 2) & 1u; break; }
       }
-      if (seen) ch += (uint32_t)((int)(Va != cin) - (int)(Va != hyp));
     }
-    if (dec_out) {  // deferred prefix decision words
+    uint32_t hi, msr, mdec, mint, ch;
+    if constexpr (kPack) {
+      hi = B.cnt_a[k] & 0xFFFFu; msr = B.cnt_a[k] >> 16;
+      mdec = B.cnt_b[k] & 0xFFFFu; mint = B.cnt_b[k] >> 16;
+      ch = B.cnt_c[k];
+    } else {
+      hi = B.cnt_a[k]; msr = B.cnt_b[k]; mdec = B.cnt_c[k]; mint = B.cnt_d[k]; ch = B.cnt_e[k];
+    }
+    unsigned long long qmin = B.qmin[k], qmax = S.qmax, dig = B.dig[k];
+    if (cin != hyp) {
+      const uint32_t n_int = seen ? (uint32_t)S.apos + 1u : (uint32_t)(t1 - t0);
+      const uint32_t n_dec = seen ? (uint32_t)S.apos : (uint32_t)(t1 - t0);
+      if (hyp) {  // assumed min, truly max
+        mint -= n_int; mdec -= n_dec;
+        qmin -= B.pqmin[k]; qmax += S.pqmax; dig -= S.pdig;
+      } else {    // assumed max, truly min
+        mint += n_int; mdec += n_dec;
+        qmin += B.pqmin[k]; qmax -= S.pqmax; dig += S.pdig;
+      }
+      const uint32_t va = (B.va >> k) & 1u;
+      if (seen) ch += (uint32_t)((int)(va != cin) - (int)(va != hyp));
+    }
+    if (want_dec) {  // deferred prefix decision words
+      uint32_t* dec_out = wk.dec + (int64_t)c * wk.dec_cstride + n;
       const uint32_t fill = cin ? ~0u : 0u;
-      const int64_t wlast = seen ? wa : wend;
+      const int64_t wlast = seen ? wt0 + S.wa : wend;
       for (int64_t w = wt0; w < wlast; ++w) dec_out[w * N] = fill & tail_mask(w * 32, T);
-      if (seen) dec_out[wa * N] = (Dwa & ~pre_dec_a) | (fill & pre_dec_a);
+      if (seen) dec_out[(wt0 + S.wa) * N] = (S.dwa & ~S.pre_dec_a) | (fill & S.pre_dec_a);
     }
     // segment sums -> per-(config, trace) accumulators (exact integer atomics)
     unsigned long long* acc = wk.acc + (int64_t)c * kAccFields * N + n;
     atomicAdd(acc + 0 * N, (unsigned long long)ev);
     atomicAdd(acc + 1 * N, (unsigned long long)hi);
     atomicAdd(acc + 2 * N, (unsigned long long)msr);
-    atomicAdd(acc + 3 * N, (unsigned long long)(int64_t)(int32_t)ch);
-    atomicAdd(acc + 4 * N, (unsigned long long)(int64_t)(int32_t)mdec);
-    atomicAdd(acc + 5 * N, (unsigned long long)(int64_t)(int32_t)mint);
+    atomicAdd(acc + 3 * N, (unsigned long long)ch);
+    atomicAdd(acc + 4 * N, (unsigned long long)mdec);
+    atomicAdd(acc + 5 * N, (unsigned long long)mint);
     atomicAdd(acc + 6 * N, qmin);
     atomicAdd(acc + 7 * N, qmax);
     atomicAdd(acc + 8 * N, qbase);
@@ -484,67 +573,73 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
   }
   __threadfence();
   consumer_sync();
-  if (tid == 0) sh_last = (atomicAdd(wk.arrive + (int64_t)c * ngroups + g, 1u) == (uint32_t)(nseg - 1));
+  if (tid == 0) sh_last = (atomicAdd(wk.arrive + (int64_t)c0 * ngroups + g, 1u) == (uint32_t)(nseg - 1));
   consumer_sync();
-  if (sh_last) {  // all segments of (config c, group g) are in: finalise the 128 traces
+  if (sh_last) {  // all segments of (bundle, group g) are in: finalise the 128 traces
     __threadfence();
-    unsigned long long tv[kTotAcc];
+#pragma unroll 1
+    for (int k = 0; k < NB; ++k) {
+      const int32_t c = cfg[k];
+      if (c < 0) continue;  // uniform across the CTA
+      unsigned long long tv[kTotAcc];
 #pragma unroll
-    for (int k = 0; k < kTotAcc; ++k) tv[k] = 0;
-    if (valid) {
-      unsigned long long* acc = wk.acc + (int64_t)c * kAccFields * N + n;
-      unsigned long long a[kAccFields];
+      for (int q = 0; q < kTotAcc; ++q) tv[q] = 0;
+      if (valid) {
+        unsigned long long* acc = wk.acc + (int64_t)c * kAccFields * N + n;
+        unsigned long long a[kAccFields];
 #pragma unroll
-      for (int k = 0; k < kAccFields; ++k) {
-        a[k] = __ldcg(acc + k * N);
-        acc[k * N] = 0ULL;  // self-cleaning for the next replay
+        for (int q = 0; q < kAccFields; ++q) {
+          a[q] = __ldcg(acc + q * N);
+          acc[q * N] = 0ULL;  // self-cleaning for the next replay
+        }
+        magus_summary sm_out;
+        finalize_summary(plat, T, (int64_t)a[0], (int64_t)a[1], (int64_t)a[2], (int64_t)a[3],
+                         (int64_t)a[4], (int64_t)a[5], a[6], a[7], a[8], a[9], &sm_out,
+                         (wk.base && c == 0) ? wk.base + n : nullptr);
+        if (wk.summary) wk.summary[(int64_t)c * N + n] = sm_out;
+        tv[0] = (unsigned long long)sm_out.viol;
+#pragma unroll
+        for (int q = 0; q < 6; ++q) tv[1 + q] = a[q];
+        tv[7] = a[6] & 0xFFFFFFFFULL; tv[8] = a[6] >> 32;
+        tv[9] = a[7] & 0xFFFFFFFFULL; tv[10] = a[7] >> 32;
+        tv[11] = a[8] & 0xFFFFFFFFULL; tv[12] = a[8] >> 32;
       }
-      magus_summary sm_out;
-      finalize_summary(plat, T, (int64_t)a[0], (int64_t)a[1], (int64_t)a[2], (int64_t)a[3],
-                       (int64_t)a[4], (int64_t)a[5], a[6], a[7], a[8], a[9], &sm_out,
-                       (wk.base && c == 0) ? wk.base + n : nullptr);
-      if (wk.summary) wk.summary[(int64_t)c * N + n] = sm_out;
-      tv[0] = (unsigned long long)sm_out.viol;
+      if (wk.totals) {  // per-config fleet totals (exact integer sums)
 #pragma unroll
-      for (int k = 0; k < 6; ++k) tv[1 + k] = a[k];
-      tv[7] = a[6] & 0xFFFFFFFFULL; tv[8] = a[6] >> 32;
-      tv[9] = a[7] & 0xFFFFFFFFULL; tv[10] = a[7] >> 32;
-      tv[11] = a[8] & 0xFFFFFFFFULL; tv[12] = a[8] >> 32;
-    }
-    if (wk.totals) {  // per-config fleet totals (exact integer sums)
+        for (int q = 0; q < kTotAcc; ++q) {
+          unsigned long long v = tv[q];
 #pragma unroll
-      for (int k = 0; k < kTotAcc; ++k) {
-        unsigned long long v = tv[k];
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xFFFFFFFFu, v, o);
-        if (lane == 0) sh_red[warp][k] = v;
-      }
-      consumer_sync();
-      if (tid < kTotAcc) {
-        unsigned long long v = 0;
-        for (int q = 0; q < kConsumerWarps; ++q) v += sh_red[q][tid];
-        atomicAdd(wk.tacc + (int64_t)c * kTotAcc + tid, v);
-      }
-      __threadfence();
-      consumer_sync();
-      if (tid == 0) sh_last2 = (atomicAdd(wk.tarrive + c, 1u) == (uint32_t)(ngroups - 1));
-      consumer_sync();
-      if (sh_last2) {
-        __threadfence();
-        uint64_t* out = wk.totals + (int64_t)c * MAGUS_TOT_WORDS;
+          for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xFFFFFFFFu, v, o);
+          if (lane == 0) sh_red[warp][q] = v;
+        }
+        consumer_sync();
         if (tid < kTotAcc) {
-          out[1 + tid] = __ldcg(wk.tacc + (int64_t)c * kTotAcc + tid);
-          wk.tacc[(int64_t)c * kTotAcc + tid] = 0ULL;
+          unsigned long long v = 0;
+          for (int q = 0; q < kConsumerWarps; ++q) v += sh_red[q][tid];
+          atomicAdd(wk.tacc + (int64_t)c * kTotAcc + tid, v);
         }
-        if (tid == 0) {
-          out[MAGUS_TOT_N_TRACES] = (uint64_t)N;
-          out[MAGUS_TOT_N_STEPS] = (uint64_t)N * (uint64_t)T;
-          out[MAGUS_TOT_RESERVED] = 0;
-          wk.tarrive[c] = 0;
+        __threadfence();
+        consumer_sync();
+        if (tid == 0) sh_last2 = (atomicAdd(wk.tarrive + c, 1u) == (uint32_t)(ngroups - 1));
+        consumer_sync();
+        if (sh_last2) {
+          __threadfence();
+          uint64_t* out = wk.totals + (int64_t)c * MAGUS_TOT_WORDS;
+          if (tid < kTotAcc) {
+            out[1 + tid] = __ldcg(wk.tacc + (int64_t)c * kTotAcc + tid);
+            wk.tacc[(int64_t)c * kTotAcc + tid] = 0ULL;
+          }
+          if (tid == 0) {
+            out[MAGUS_TOT_N_TRACES] = (uint64_t)N;
+            out[MAGUS_TOT_N_STEPS] = (uint64_t)N * (uint64_t)T;
+            out[MAGUS_TOT_RESERVED] = 0;
+            wk.tarrive[c] = 0;
+          }
         }
+        consumer_sync();  // sh_red / sh_last2 are reused by the next config
       }
     }
-    if (tid == 0) wk.arrive[(int64_t)c * ngroups + g] = 0;
+    if (tid == 0) wk.arrive[(int64_t)c0 * ngroups + g] = 0;
   }
   if (tid == 0) {  // the last CTA of the launch re-arms the ticket counter
     __threadfence();
@@ -563,27 +658,37 @@ struct Pick {
   int smem;
 };
 
-Pick pick(int32_t W, int32_t H) {
+template <int NB>
+Pick pick_nb(int32_t W, int32_t H) {
   if (H == 10) {
     switch (W) {
-      case 4: return {stream_kernel<4, 10>, Stages<4>::smem};
-      case 6: return {stream_kernel<6, 10>, Stages<6>::smem};
-      case 10: return {stream_kernel<10, 10>, Stages<10>::smem};
-      case 16: return {stream_kernel<16, 10>, Stages<16>::smem};
+      case 4: return {stream_kernel<4, 10, NB>, Stages<4>::smem};
+      case 6: return {stream_kernel<6, 10, NB>, Stages<6>::smem};
+      case 10: return {stream_kernel<10, 10, NB>, Stages<10>::smem};
+      case 16: return {stream_kernel<16, 10, NB>, Stages<16>::smem};
       default: break;
     }
-    if (W >= 2 && W <= 33) return {stream_kernel<0, 10>, Stages<0>::smem};
+    if (W >= 2 && W <= 33) return {stream_kernel<0, 10, NB>, Stages<0>::smem};
   }
-  if (W >= 2 && W <= 33 && H >= 1 && H <= 32) return {stream_kernel<0, 0>, Stages<0>::smem};
+  if (W >= 2 && W <= 33 && H >= 1 && H <= 32) return {stream_kernel<0, 0, NB>, Stages<0>::smem};
   return {nullptr, 0};
+}
+
+Pick pick(int32_t W, int32_t H, int32_t NB) {
+  switch (NB) {
+    case 1: return pick_nb<1>(W, H);
+    case 2: return pick_nb<2>(W, H);
+    case 4: return pick_nb<4>(W, H);
+    default: return {nullptr, 0};
+  }
 }
 
 }  // namespace
 
-bool stream_supported(int32_t W, int32_t H) { return pick(W, H).f != nullptr; }
+bool stream_supported(int32_t W, int32_t H) { return pick(W, H, 1).f != nullptr; }
 
-int stream_ctas_per_sm(int32_t W, int32_t H) {
-  Pick p = pick(W, H);
+int stream_ctas_per_sm(int32_t W, int32_t H, int32_t NB) {
+  Pick p = pick(W, H, NB);
   if (!p.f) return 0;
   cudaFuncSetAttribute((const void*)p.f, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem);
   int nb = 0;
@@ -594,18 +699,18 @@ int stream_ctas_per_sm(int32_t W, int32_t H) {
 }
 
 int launch_stream(cudaStream_t st, const void* tmap, int64_t N, int64_t T,
-                  const DevPolicy* pol_dev, const int32_t* cidx_dev, int32_t nc, int32_t W,
-                  int32_t H, const DevPlatform& plat, int64_t nseg, int64_t seg_len,
+                  const DevPolicy* pol_dev, const int32_t* bundles_dev, int32_t nbund, int32_t NB,
+                  int32_t W, int32_t H, const DevPlatform& plat, int64_t nseg, int64_t seg_len,
                   const StreamWork& wk, int* grid_out) {
-  Pick p = pick(W, H);
+  Pick p = pick(W, H, NB);
   if (!p.f) return -1;
   cudaFuncSetAttribute((const void*)p.f, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem);
   const int32_t ngroups = (int32_t)((N + kTraces - 1) / kTraces);
-  const int64_t grid = (int64_t)ngroups * nseg * nc;
+  const int64_t grid = (int64_t)ngroups * nseg * nbund;
   if (grid_out) *grid_out = (int)grid;
   const CUtensorMap* m = reinterpret_cast<const CUtensorMap*>(tmap);
-  p.f<<<(unsigned)grid, kThreads, p.smem, st>>>(*m, N, T, pol_dev, cidx_dev, plat, nseg, seg_len,
-                                                ngroups, nc, wk);
+  p.f<<<(unsigned)grid, kThreads, p.smem, st>>>(*m, N, T, pol_dev, bundles_dev, plat, nseg, seg_len,
+                                                ngroups, nbund, wk);
   return cudaGetLastError() == cudaSuccess ? 1 : -1;
 }
 

@@ -78,13 +78,15 @@ int launch_reference(cudaStream_t s, const float* x, int64_t N, int64_t T, int64
                      magus_summary* out_summary, magus_base* out_base, uint32_t* out_dec);
 
 bool stream_supported(int32_t W, int32_t H);
-// Fused stream kernel over the nc configs listed in cidx_dev (global indices;
-// all share (W, H)): replay + carry look-back + finalisation + totals.
+// Fused stream kernel over nbund bundles of NB configs (bundles_dev:
+// [nbund][NB] global config indices, -1 = padding).  All configs of a launch
+// share (W, H); the configs of a bundle also share L, tau_inc and tau_dec.
+// Replay + carry look-back + finalisation + totals in one launch.
 int launch_stream(cudaStream_t s, const void* tmap /* CUtensorMap, host copy */, int64_t N,
-                  int64_t T, const DevPolicy* pol_dev, const int32_t* cidx_dev, int32_t nc,
-                  int32_t W, int32_t H, const DevPlatform& plat, int64_t nseg, int64_t seg_len,
-                  const StreamWork& wk, int* grid_out);
-int stream_ctas_per_sm(int32_t W, int32_t H);
+                  int64_t T, const DevPolicy* pol_dev, const int32_t* bundles_dev, int32_t nbund,
+                  int32_t NB, int32_t W, int32_t H, const DevPlatform& plat, int64_t nseg,
+                  int64_t seg_len, const StreamWork& wk, int* grid_out);
+int stream_ctas_per_sm(int32_t W, int32_t H, int32_t NB);
 
 int launch_totals(cudaStream_t s, const magus_summary* summary, const magus_base* base, int64_t N,
                   int64_t T, int32_t C, uint64_t* totals);

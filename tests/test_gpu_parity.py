@@ -253,3 +253,23 @@ def test_full_config2_sampled_parity(ctx):
         ctx.set_option(magus.OPT_KERNEL, magus.KERNEL_AUTO)
     assert np.array_equal(r2.summary_numpy(), got)
     assert np.array_equal(r2.totals_numpy(), r.totals_numpy())
+
+
+@pytest.mark.parametrize("bundle", [0, 1, 2, 4])
+def test_bundles_share_alg1_alg2_work_exactly(ctx, bundle):
+    """Configs differing only in t_hi share Delta, events and the window count
+    (one thread, NB configs); padding and any NB give identical results."""
+    N, T = 200, 2600
+    x = gen.gen_traces(gen.SEEDS[3], N, T)
+    pols = [magus.make_policy(W=10, tau_inc=ti, tau_dec=td, t_hi=th)
+            for (ti, td) in [(200, -500), (100, -250)] for th in (0.2, 0.3, 0.4, 0.5, 0.7)]
+    pols += [magus.make_policy(W=6, tau_inc=300, tau_dec=-750, t_hi=th) for th in (0.1, 0.4, 1.5)]
+    pols += [magus.make_policy(W=7, H=13, L=3.0, tau_inc=90, tau_dec=-90, t_hi=th) for th in (0.25, 0.5)]
+    ref = oracle.replay(x, to_oracle_policies(pols), want_dec=True)
+    ctx.set_option(magus.OPT_BUNDLE, bundle)
+    try:
+        for segments in (0, 7):
+            r = run_gpu(ctx, x, pols, magus.KERNEL_STREAM, segments=segments)
+            assert_parity(r, ref, pols, T)
+    finally:
+        ctx.set_option(magus.OPT_BUNDLE, 0)
