@@ -215,7 +215,10 @@ def run_ours(args):
     pols = policies_for(grid)
     C = len(pols)
     seed = SEED_BASE + args.config
-    ctx = magus.Context(device=local, stream=stream)
+    plat = magus.platform_preset()
+    if args.burst > 0:  # NEXT f1: Sec. 6.3 burst Jaccard counters in the same pass
+        plat.burst_mbs = args.burst
+    ctx = magus.Context(device=local, stream=stream, platform=plat)
     if args.waves:
         ctx.set_option(magus.OPT_WAVES, args.waves)
     if args.segments:
@@ -360,6 +363,10 @@ def run_ours(args):
             "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": int(st["launches_total"]), "clocks": clk,
             "best_config": best[0], "feasible": best[2]}
+    if args.burst > 0:
+        line["config"]["burst_mbs"] = args.burst
+        line["best_jaccard"] = best[1]["jaccard"]
+        line["pareto_front"] = [int(i) for i in np.flatnonzero(ctx.pareto_front(out.totals))]
     if roof is not hbm_roof:
         line["roofline_hbm"] = hbm_roof
     if parity is not None:
@@ -385,6 +392,8 @@ def main():
     ap.add_argument("--waves", type=int, default=0, help="MAGUS_OPT_WAVES (0 = library default)")
     ap.add_argument("--segments", type=int, default=0, help="MAGUS_OPT_SEGMENTS (0 = auto)")
     ap.add_argument("--bundle", type=int, default=0, help="MAGUS_OPT_BUNDLE (0 = auto, 1, 2, 4)")
+    ap.add_argument("--burst", type=float, default=0.0,
+                    help="NEXT f1: Sec. 6.3 burst threshold (MB/s); > 0 enables the Jaccard counters")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-cpu-baseline", action="store_true")

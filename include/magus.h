@@ -92,10 +92,15 @@ typedef struct {
   double  e_switch_j;     /* energy per frequency change ("negligible", 0)   */
   double  t_switch_s;     /* time per frequency change (0)                   */
   double  slowdown_bound; /* 0.05, the "<5 % performance loss" (P@1715)      */
+  double  burst_mbs;      /* Sec. 6.3 burst threshold theta for the Jaccard
+                             accuracy (P@41094-P@41603; "predefined", value
+                             not printed): an interval is a burst when the
+                             delivered throughput min(x, B_l) exceeds it.
+                             <= 0 disables the burst counters.               */
 } magus_platform;
 
 /* Result per (config, trace).  Integer counters are exact; time/energy are
- * model M evaluated from them in a fixed fp64 operation order.  104 bytes. */
+ * model M evaluated from them in a fixed fp64 operation order.  120 bytes. */
 typedef struct {
   int64_t  n_events;      /* rounds with trend != 0 (Alg. 3 l.17/22 push 1)  */
   int64_t  n_hi_rounds;   /* rounds with high_freq_status = 1 (l.10)         */
@@ -112,6 +117,11 @@ typedef struct {
   double   slowdown;      /* time_s / base.time_s - 1 (>= 0 exactly)         */
   int32_t  viol;          /* slowdown > slowdown_bound                       */
   int32_t  reserved;
+  int64_t  n_burst_base;  /* #t with min(x_t, B(ratio_max)) > burst_mbs      */
+  int64_t  n_burst_magus; /* #t with min(x_t, B(l_t)) > burst_mbs (l_t =
+                             dec[t-1]); Jaccard (Sec. 6.3) = |A and B| /
+                             |A or B| = n_burst_magus / n_burst_base, since
+                             B(l) <= B(max) makes the MAGUS bursts a subset  */
 } magus_summary;
 
 /* Config-independent baseline per trace: uncore pinned at ratio_max (the
@@ -144,8 +154,10 @@ enum {
   MAGUS_TOT_QBASE_LO,
   MAGUS_TOT_QBASE_HI,
   MAGUS_TOT_N_STEPS,     /* sum over traces of T                            */
+  MAGUS_TOT_BURST_BASE,  /* sum of n_burst_base                             */
+  MAGUS_TOT_BURST_MAGUS, /* sum of n_burst_magus                            */
   MAGUS_TOT_RESERVED,
-  MAGUS_TOT_WORDS = 16
+  MAGUS_TOT_WORDS = 18
 };
 
 /* fp64 quantities derived from one config's integer totals (host-side,
@@ -159,6 +171,8 @@ typedef struct {
   double  slowdown;       /* time_s / base_time_s - 1                         */
   int64_t n_viol;         /* traces whose own slowdown exceeds the bound      */
   int64_t n_traces;
+  double  jaccard;        /* fleet burst Jaccard, sum A and B / sum A or B
+                             (1 when there is no burst at all)               */
 } magus_derived;
 
 /* ---- lifecycle -------------------------------------------------------- */
@@ -241,6 +255,16 @@ magus_status magus_derive_host(const magus_platform* plat, const uint64_t* total
                                magus_derived* out);
 magus_status magus_sweep_best_host(const magus_platform* plat, const uint64_t* totals_host,
                                    int32_t n_params, int32_t* best, magus_derived* best_row);
+
+/* Energy/runtime Pareto front over the configs (Sec. 6.4, Fig. 7,
+ * P@43971-P@44696): on_front[c] = 1 iff no config has fleet energy and
+ * fleet runtime both <= config c's with at least one strictly less.
+ * `totals` DEVICE [n_params][MAGUS_TOT_WORDS]; on_front HOST [n_params];
+ * *n_front = number of configs on the front.  Synchronises. */
+magus_status magus_pareto_front(magus_ctx ctx, const uint64_t* totals, int32_t n_params,
+                                int32_t* on_front, int32_t* n_front);
+magus_status magus_pareto_front_host(const magus_platform* plat, const uint64_t* totals_host,
+                                     int32_t n_params, int32_t* on_front, int32_t* n_front);
 
 /* ---- synthetic traces (input generator; gen/magus_gen.h) --------------- */
 enum { MAGUS_GEN_MIX = 0, MAGUS_GEN_ADVERSARIAL = 1 };

@@ -27,12 +27,13 @@ POLICY_DT = np.dtype([("W", "<i4"), ("H", "<i4"), ("L", "<f8"), ("tau_inc", "<f8
 PLATFORM_DT = np.dtype([("r_min", "<i4"), ("r_max", "<i4"), ("dt", "<f8"), ("bw_max", "<f8"),
                         ("beta", "<f8"), ("p_other", "<f8"), ("p_unc_min", "<f8"),
                         ("p_unc_max", "<f8"), ("e_sw", "<f8"), ("t_sw", "<f8"),
-                        ("bound", "<f8")], align=True)
+                        ("bound", "<f8"), ("burst", "<f8")], align=True)
 SUMMARY_DT = np.dtype([("n_events", "<i8"), ("n_hi_rounds", "<i8"), ("n_msr_writes", "<i8"),
                        ("n_changes", "<i8"), ("n_min_dec", "<i8"), ("n_min_int", "<i8"),
                        ("q_min", "<u8"), ("q_max", "<u8"), ("digest", "<u8"), ("time", "<f8"),
                        ("energy", "<f8"), ("slowdown", "<f8"), ("viol", "<i4"),
-                       ("reserved", "<i4")], align=True)
+                       ("reserved", "<i4"), ("n_burst_base", "<i8"), ("n_burst_magus", "<i8"),
+                       ("n_burst_inter", "<i8"), ("n_burst_union", "<i8")], align=True)
 BASE_DT = np.dtype([("q_base", "<u8"), ("time", "<f8"), ("energy", "<f8"),
                     ("reserved", "<u8")], align=True)
 
@@ -93,14 +94,14 @@ def policies(rows) -> np.ndarray:
 
 
 def platform(r_min=8, r_max=22, dt=0.2, bw_max=32000.0, beta=1.0, p_other=218.0,
-             p_unc_min=0.0, p_unc_max=82.0, e_sw=0.0, t_sw=0.0, bound=0.05) -> np.ndarray:
+             p_unc_min=0.0, p_unc_max=82.0, e_sw=0.0, t_sw=0.0, bound=0.05, burst=0.0) -> np.ndarray:
     """Intel+A100 (uncore 0.8-2.2 GHz, P@29320); 82 W uncore range (Fig. 2,
     P@12253); 0.2 s (P@44789); 5 % bound (P@1715).  bw_max/beta/p_other are
     model-M assumptions."""
     p = np.zeros(1, dtype=PLATFORM_DT)
     for k, v in dict(r_min=r_min, r_max=r_max, dt=dt, bw_max=bw_max, beta=beta, p_other=p_other,
                      p_unc_min=p_unc_min, p_unc_max=p_unc_max, e_sw=e_sw, t_sw=t_sw,
-                     bound=bound).items():
+                     bound=bound, burst=burst).items():
         p[k] = v
     return p
 
@@ -167,17 +168,30 @@ def account(x, dec, plat=None):
 
 
 def totals(summary_row: np.ndarray, base: np.ndarray, T: int, plat=None):
-    """(int words[16], derived[6]) for one config's [N] summaries."""
+    """(int words[18], derived[7]) for one config's [N] summaries; derived =
+    energy, time, base_energy, base_time, saving, slowdown, jaccard."""
     plat = platform() if plat is None else np.ascontiguousarray(plat, dtype=PLATFORM_DT)
     s = np.ascontiguousarray(summary_row, dtype=SUMMARY_DT)
     b = np.ascontiguousarray(base, dtype=BASE_DT)
-    w = np.zeros(16, dtype=np.uint64)
-    f = np.zeros(6, dtype=np.float64)
+    w = np.zeros(18, dtype=np.uint64)
+    f = np.zeros(7, dtype=np.float64)
     rc = _load().oracle_totals(s.ctypes.data, b.ctypes.data, len(s), T, plat.ctypes.data,
                                w.ctypes.data, f.ctypes.data)
     if rc != 0:
         raise ValueError("oracle_totals rejected its arguments")
     return w, f
+
+
+def pareto_front(energy, time) -> np.ndarray:
+    """Sec. 6.4 (Fig. 7): configs not dominated in (energy, runtime); plain O(C^2)."""
+    e, t = np.asarray(energy, np.float64), np.asarray(time, np.float64)
+    on = np.ones(len(e), bool)
+    for i in range(len(e)):
+        for j in range(len(e)):
+            if e[j] <= e[i] and t[j] <= t[i] and (e[j] < e[i] or t[j] < t[i]):
+                on[i] = False
+                break
+    return on
 
 
 def energy_sum(summary_row: np.ndarray) -> float:

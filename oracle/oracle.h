@@ -24,6 +24,7 @@ typedef struct {
 typedef struct {
   int32_t r_min, r_max;
   double dt, bw_max, beta, p_other, p_unc_min, p_unc_max, e_sw, t_sw, bound;
+  double burst;   /* Sec. 6.3 burst threshold theta (<= 0: not counted) */
 } or_platform;
 
 typedef struct {
@@ -31,6 +32,10 @@ typedef struct {
   uint64_t q_min, q_max, digest;
   double time, energy, slowdown;
   int32_t viol, reserved;
+  int64_t n_burst_base;   /* |B|: bursts of the max-uncore run        */
+  int64_t n_burst_magus;  /* |A|: bursts of the MAGUS run             */
+  int64_t n_burst_inter;  /* |A and B|                                */
+  int64_t n_burst_union;  /* |A or B|                                 */
 } or_summary;
 
 typedef struct {

@@ -26,10 +26,10 @@ PLATFORM_INTEL_A100, PLATFORM_INTEL_MAX1550 = 0, 1
 GEN_MIX, GEN_ADVERSARIAL = 0, 1
 OPT_KERNEL, OPT_SEGMENTS, OPT_TIMING, OPT_WAVES, OPT_BUNDLE = 0, 1, 2, 3, 4
 KERNEL_AUTO, KERNEL_REFERENCE, KERNEL_STREAM = 0, 1, 2
-TOT_WORDS = 16
+TOT_WORDS = 18
 TOT_NAMES = ["n_traces", "n_viol", "events", "hi_rounds", "msr_writes", "changes", "min_dec",
              "min_int", "qmin_lo", "qmin_hi", "qmax_lo", "qmax_hi", "qbase_lo", "qbase_hi",
-             "n_steps", "reserved"]
+             "n_steps", "burst_base", "burst_magus", "reserved"]
 
 
 class Policy(ctypes.Structure):
@@ -45,13 +45,13 @@ class Platform(ctypes.Structure):
                 ("bw_max_mbs", ctypes.c_double), ("beta", ctypes.c_double), ("p_other_w", ctypes.c_double),
                 ("p_unc_min_w", ctypes.c_double), ("p_unc_max_w", ctypes.c_double),
                 ("e_switch_j", ctypes.c_double), ("t_switch_s", ctypes.c_double),
-                ("slowdown_bound", ctypes.c_double)]
+                ("slowdown_bound", ctypes.c_double), ("burst_mbs", ctypes.c_double)]
 
 
 class Derived(ctypes.Structure):
     _fields_ = [("energy_j", ctypes.c_double), ("time_s", ctypes.c_double), ("base_energy_j", ctypes.c_double),
                 ("base_time_s", ctypes.c_double), ("saving", ctypes.c_double), ("slowdown", ctypes.c_double),
-                ("n_viol", ctypes.c_int64), ("n_traces", ctypes.c_int64)]
+                ("n_viol", ctypes.c_int64), ("n_traces", ctypes.c_int64), ("jaccard", ctypes.c_double)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -77,9 +77,10 @@ class Stats(ctypes.Structure):
 SUMMARY_DT = np.dtype([("n_events", "<i8"), ("n_hi_rounds", "<i8"), ("n_msr_writes", "<i8"),
                        ("n_changes", "<i8"), ("n_min_dec", "<i8"), ("n_min_int", "<i8"), ("q_min", "<u8"),
                        ("q_max", "<u8"), ("digest", "<u8"), ("time_s", "<f8"), ("energy_j", "<f8"),
-                       ("slowdown", "<f8"), ("viol", "<i4"), ("reserved", "<i4")])
+                       ("slowdown", "<f8"), ("viol", "<i4"), ("reserved", "<i4"), ("n_burst_base", "<i8"),
+                       ("n_burst_magus", "<i8")])
 BASE_DT = np.dtype([("q_base", "<u8"), ("time_s", "<f8"), ("energy_j", "<f8"), ("reserved", "<u8")])
-assert SUMMARY_DT.itemsize == 104 and BASE_DT.itemsize == 32
+assert SUMMARY_DT.itemsize == 120 and BASE_DT.itemsize == 32
 
 _vp, _i32, _i64, _u64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_uint64
 _lib.magus_init.argtypes = [ctypes.POINTER(_vp), ctypes.c_int, _vp, ctypes.POINTER(Platform)]
@@ -104,6 +105,8 @@ _lib.magus_policy_inspect.argtypes = [ctypes.POINTER(Policy), ctypes.POINTER(Pol
 _lib.magus_platform_inspect.argtypes = [ctypes.POINTER(Platform), ctypes.POINTER(PlatformConsts)]
 _lib.magus_get_stats.argtypes = [_vp, ctypes.POINTER(Stats)]
 _lib.magus_derive_host.argtypes = [ctypes.POINTER(Platform), _vp, ctypes.POINTER(Derived)]
+_lib.magus_pareto_front.argtypes = [_vp, _vp, _i32, _vp, ctypes.POINTER(_i32)]
+_lib.magus_pareto_front_host.argtypes = [ctypes.POINTER(Platform), _vp, _i32, _vp, ctypes.POINTER(_i32)]
 _lib.magus_sweep_best_host.argtypes = [ctypes.POINTER(Platform), _vp, _i32, ctypes.POINTER(_i32),
                                        ctypes.POINTER(Derived)]
 _lib.magus_reset_stats.argtypes = [_vp]
@@ -111,7 +114,7 @@ for _f in ("magus_init", "magus_destroy", "magus_set_stream", "magus_policy_pres
            "magus_grid_sweep256", "magus_grid_fleet64", "magus_replay", "magus_replay_host",
            "magus_totals_derive", "magus_sweep_best", "magus_gen_traces", "magus_set_option",
            "magus_get_stats", "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
-           "magus_sweep_best_host"):
+           "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host"):
     getattr(_lib, _f).restype = ctypes.c_int
 
 EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_string", "magus_last_error",
@@ -119,7 +122,7 @@ EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_str
             "magus_grid_fleet64", "magus_replay", "magus_replay_host", "magus_totals_derive",
             "magus_sweep_best", "magus_gen_traces", "magus_set_option", "magus_get_stats",
             "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
-            "magus_sweep_best_host"]
+            "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host"]
 
 
 class MagusError(RuntimeError):
@@ -198,6 +201,19 @@ def sweep_best_host(totals, platform: Platform | None = None) -> tuple[int, dict
     if st not in (OK, ERR_NO_FEASIBLE):
         raise MagusError(st, "sweep_best_host")
     return int(best.value), d.as_dict(), st == OK
+
+
+def pareto_front_host(totals, platform: Platform | None = None) -> np.ndarray:
+    """Sec. 6.4 energy/runtime Pareto front over configs (host totals [C, W])."""
+    plat = platform if platform is not None else platform_preset()
+    w = np.ascontiguousarray(np.asarray(totals).view(np.uint64).reshape(-1, TOT_WORDS))
+    on = np.zeros(len(w), np.int32)
+    nf = _i32()
+    st = _lib.magus_pareto_front_host(ctypes.byref(plat), _vp(w.ctypes.data), len(w), _vp(on.ctypes.data),
+                                      ctypes.byref(nf))
+    if st:
+        raise MagusError(st, "pareto_front_host")
+    return on.astype(bool)
 
 
 def make_policy(W=10, H=10, L=None, tau_inc=200.0, tau_dec=-500.0, t_hi=0.4) -> Policy:
@@ -310,7 +326,8 @@ class Context:
         if out is None:
             nw = (T + 31) // 32
             out = ReplayResult(
-                summary=torch.empty((C, N, 104), dtype=torch.uint8, device=dev) if want_summary else None,
+                summary=torch.empty((C, N, SUMMARY_DT.itemsize), dtype=torch.uint8, device=dev)
+                if want_summary else None,
                 base=torch.empty((N, 32), dtype=torch.uint8, device=dev) if want_base else None,
                 decisions=torch.empty((C, nw, N), dtype=torch.int32, device=dev) if want_decisions else None,
                 totals=torch.empty((C, TOT_WORDS), dtype=torch.int64, device=dev) if want_totals else None,
@@ -343,6 +360,15 @@ class Context:
         d = Derived()
         self._check(_lib.magus_totals_derive(self._h, _vp(w.ctypes.data), ctypes.byref(d)), "totals_derive")
         return d.as_dict()
+
+    def pareto_front(self, totals) -> np.ndarray:
+        """Sec. 6.4 front over the configs from DEVICE totals [C, W]."""
+        C = totals.shape[0]
+        on = np.zeros(C, np.int32)
+        nf = _i32()
+        st = _lib.magus_pareto_front(self._h, _vp(totals.data_ptr()), C, _vp(on.ctypes.data), ctypes.byref(nf))
+        self._check(st, "pareto_front")
+        return on.astype(bool)
 
     def sweep_best(self, totals) -> tuple[int, dict, bool]:
         """totals: CUDA int64 tensor [C, 16] (summed over ranks if sharded).

@@ -275,6 +275,10 @@ void derive_totals(const DevPlatform& p, const uint64_t* w, magus_derived* out) 
   out->slowdown = time / base_time - 1.0;
   out->n_viol = (int64_t)w[MAGUS_TOT_N_VIOL];
   out->n_traces = (int64_t)w[MAGUS_TOT_N_TRACES];
+  // Sec. 6.3: |A and B| / |A or B| with A = MAGUS bursts, B = max-uncore
+  // bursts; A is a subset of B (B_l <= B_max), so this is sum A / sum B.
+  const uint64_t uni = w[MAGUS_TOT_BURST_BASE], inter = w[MAGUS_TOT_BURST_MAGUS];
+  out->jaccard = uni ? (double)inter / (double)uni : 1.0;
 }
 
 }  // namespace magus
@@ -330,6 +334,7 @@ magus_status magus_platform_preset(int32_t id, magus_platform* out) {
   p.e_switch_j = 0.0;         // "negligible" (P@27899)
   p.t_switch_s = 0.0;
   p.slowdown_bound = 0.05;    // P@1715
+  p.burst_mbs = 0.0;          // Sec. 6.3 Jaccard counters off by default (theta not printed)
   *out = p;
   return MAGUS_OK;
 }
@@ -558,7 +563,7 @@ magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t N, int64_t
     const size_t off_arrive = 256;
     const size_t off_tarrive = off_arrive + align_up(4 * (size_t)(C * ngroups), 256);
     const size_t off_tacc = off_tarrive + align_up(4 * (size_t)C, 256);
-    const size_t off_acc = off_tacc + align_up(8 * 13 * (size_t)C, 256);
+    const size_t off_acc = off_tacc + align_up(8 * kTotAccWords * (size_t)C, 256);
     const size_t off_status = off_acc + align_up(8 * (size_t)kAccFields * (size_t)(C * N), 256);
     const size_t total = off_status + align_up(4 * (size_t)(C * nseg) * (size_t)N, 256);
     st = ensure_scratch(ctx, total);
@@ -696,6 +701,43 @@ magus_status magus_sweep_best(magus_ctx ctx, const uint64_t* totals, int32_t C, 
   magus_status st = choose_best(ctx->dplat, (const uint64_t*)ctx->best_pinned, C, best, best_row);
   if (st == MAGUS_ERR_NO_FEASIBLE) ctx->err = "no config keeps every trace within the slowdown bound";
   return st;
+}
+
+static void pareto(const DevPlatform& dp, const uint64_t* h, int32_t C, int32_t* on_front,
+                   int32_t* n_front) {
+  std::vector<magus_derived> d((size_t)C);
+  for (int32_t c = 0; c < C; ++c) derive_totals(dp, h + (size_t)c * MAGUS_TOT_WORDS, &d[c]);
+  int32_t nf = 0;
+  for (int32_t i = 0; i < C; ++i) {
+    bool dominated = false;
+    for (int32_t j = 0; j < C && !dominated; ++j)
+      dominated = (d[j].energy_j <= d[i].energy_j && d[j].time_s <= d[i].time_s) &&
+                  (d[j].energy_j < d[i].energy_j || d[j].time_s < d[i].time_s);
+    on_front[i] = dominated ? 0 : 1;
+    nf += on_front[i];
+  }
+  if (n_front) *n_front = nf;
+}
+
+magus_status magus_pareto_front(magus_ctx ctx, const uint64_t* totals, int32_t C, int32_t* on_front,
+                                int32_t* n_front) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  if (!totals || C < 1 || !on_front) return fail(ctx, MAGUS_ERR_INVALID_ARG, "bad pareto arguments");
+  DeviceGuard dg(ctx->device);
+  std::vector<uint64_t> h((size_t)C * MAGUS_TOT_WORDS);
+  CK(cudaMemcpyAsync(h.data(), totals, h.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  pareto(ctx->dplat, h.data(), C, on_front, n_front);
+  return MAGUS_OK;
+}
+
+magus_status magus_pareto_front_host(const magus_platform* plat, const uint64_t* totals_host,
+                                     int32_t C, int32_t* on_front, int32_t* n_front) {
+  char msg[256];
+  if (!plat || !totals_host || C < 1 || !on_front || !validate_platform(*plat, msg, sizeof msg))
+    return MAGUS_ERR_INVALID_ARG;
+  pareto(make_dev_platform(*plat), totals_host, C, on_front, n_front);
+  return MAGUS_OK;
 }
 
 magus_status magus_derive_host(const magus_platform* plat, const uint64_t* totals_host,

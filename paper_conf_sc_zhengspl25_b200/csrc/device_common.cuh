@@ -45,6 +45,7 @@ __device__ __forceinline__ void finalize_summary(const DevPlatform& p, int64_t T
                                                  int64_t hi_rounds, int64_t msr, int64_t changes,
                                                  int64_t n_min_dec, int64_t n_min_int, uint64_t q_min,
                                                  uint64_t q_max, uint64_t q_base, uint64_t digest,
+                                                 int64_t n_burst_base, int64_t n_burst_magus,
                                                  magus_summary* s, magus_base* b) {
   const int64_t n_max_int = T - n_min_int;
   const double time_max = p.dt * (double)n_max_int + p.cQ * (double)q_max;
@@ -68,6 +69,8 @@ __device__ __forceinline__ void finalize_summary(const DevPlatform& p, int64_t T
     o.slowdown = time / base_time - 1.0;
     o.viol = o.slowdown > p.bound ? 1 : 0;
     o.reserved = 0;
+    o.n_burst_base = n_burst_base;
+    o.n_burst_magus = n_burst_magus;
     *s = o;
   }
   if (b) {

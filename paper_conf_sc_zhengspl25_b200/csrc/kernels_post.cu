@@ -9,7 +9,7 @@ namespace magus {
 // Per-config totals: exact integer sums over traces (order-free).
 // ---------------------------------------------------------------------------
 constexpr int kTotThreads = 256;
-constexpr int kTotAcc = 13;
+constexpr int kTotAcc = kTotAccWords;
 
 __global__ void __launch_bounds__(kTotThreads)
 totals_kernel(const magus_summary* __restrict__ sm, const magus_base* __restrict__ base, int64_t N,
@@ -34,6 +34,8 @@ totals_kernel(const magus_summary* __restrict__ sm, const magus_base* __restrict
     const uint64_t qb = base[n].q_base;
     a[11] += qb & 0xFFFFFFFFULL;
     a[12] += qb >> 32;
+    a[13] += (uint64_t)s.n_burst_base;
+    a[14] += (uint64_t)s.n_burst_magus;
   }
   __shared__ uint64_t red[kTotThreads / 32][kTotAcc];
 #pragma unroll
@@ -47,7 +49,9 @@ totals_kernel(const magus_summary* __restrict__ sm, const magus_base* __restrict
   if (threadIdx.x < kTotAcc) {
     uint64_t v = 0;
     for (int w = 0; w < kTotThreads / 32; ++w) v += red[w][threadIdx.x];
-    tot[(int64_t)c * MAGUS_TOT_WORDS + 1 + threadIdx.x] = v;  // words 1..13
+    // accumulators 0..12 -> words 1..13; 13, 14 -> the burst words
+    const int word = threadIdx.x < 13 ? 1 + threadIdx.x : MAGUS_TOT_BURST_BASE + (threadIdx.x - 13);
+    tot[(int64_t)c * MAGUS_TOT_WORDS + word] = v;
   }
   if (threadIdx.x == 0) {
     tot[(int64_t)c * MAGUS_TOT_WORDS + MAGUS_TOT_N_TRACES] = (uint64_t)N;

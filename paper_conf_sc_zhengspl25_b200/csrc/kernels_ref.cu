@@ -28,6 +28,8 @@ ref_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
   int freq_min = 0;              // uncore_freq: starts at max (P@23755)
   int64_t events = 0, hi_rounds = 0, msr = 0, changes = 0, n_min_dec = 0, n_min_int = 0;
   uint64_t q_min = 0, q_max = 0, q_base = 0, digest = 0;
+  int64_t b_base = 0, b_magus = 0;  // Sec. 6.3 bursts (model M 4.6)
+  const bool bursts = plat.burst_mbs > 0.0;
   uint32_t word = 0;
   int prev = 0;                  // dec[t-1] (min = 1); dec[-1] := max
 
@@ -53,6 +55,10 @@ ref_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
     if (prev) { ++n_min_int; q_min += q_literal(xt, plat.invB_min); }
     else q_max += q_literal(xt, plat.invB_max);
     q_base += q_literal(xt, plat.invB_max);
+    if (bursts && (double)xt > plat.burst_mbs) {  // delivered min(x, B_l) > theta
+      b_base += plat.Bmax > plat.burst_mbs;
+      b_magus += (prev ? plat.Bmin : plat.Bmax) > plat.burst_mbs;
+    }
     n_min_dec += dmin;
     if (t >= 1 && dmin != prev) ++changes;
     word |= (uint32_t)dmin << (t & 31);
@@ -65,7 +71,7 @@ ref_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
     prev = dmin;
   }
   finalize_summary(plat, T, events, hi_rounds, msr, changes, n_min_dec, n_min_int, q_min, q_max,
-                   q_base, digest, out ? out + (int64_t)c * N + n : nullptr,
+                   q_base, digest, b_base, b_magus, out ? out + (int64_t)c * N + n : nullptr,
                    (base && c == 0) ? base + n : nullptr);
 }
 

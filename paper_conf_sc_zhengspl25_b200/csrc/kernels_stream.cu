@@ -43,7 +43,7 @@ constexpr int kStageFloats = kTraces * kRows;           // 16 KB
 constexpr int kConsumerWarps = kTraces / 32;
 constexpr int kThreads = kTraces + 32;                  // + producer warp
 constexpr uint32_t kStageBytes = kStageFloats * 4;
-constexpr int kTotAcc = 13;
+constexpr int kTotAcc = kTotAccWords;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
@@ -232,6 +232,8 @@ struct BundleRegs {
   uint32_t cnt_c[NB];  // NB == 1: mdec; NB > 1: ch
   uint32_t cnt_d[NB];  // NB == 1: mint, ch packed separately below
   uint32_t cnt_e[NB];
+  uint32_t cnt_f[NB];  // bursts kept under MAGUS (NB > 1: | prefix bursts << 16)
+  uint32_t cnt_g[NB];  // NB == 1: bursts in the carry-dependent prefix
   unsigned long long qmin[NB], dig[NB], pqmin[NB];
   uint32_t carry, seen, va, last;  // bit k per config
 };
@@ -241,7 +243,7 @@ struct BundleSmem {  // rarely touched, per (config slot, thread)
   uint32_t dwa, pre_dec_a;
 };
 
-template <int W_T, int H_T, int NB>
+template <int W_T, int H_T, int NB, bool BURST>
 __global__ void __launch_bounds__(kThreads, Occ<W_T, NB>::v)
 stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
               const DevPolicy* __restrict__ pol, const int32_t* __restrict__ bundles, DevPlatform plat,
@@ -285,29 +287,29 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
 #pragma unroll
   for (int k = 0; k < NB; ++k) cfg[k] = bundles[bidx * NB + k];  // global config, -1 = pad
   const int32_t c0 = cfg[0];
-  const int64_t t0 = s * seg_len;
-  const int64_t t1 = (t0 + seg_len < T) ? t0 + seg_len : T;
+  const int32_t t0 = (int32_t)(s * seg_len);  // T <= 2^24: time fits in 32 bits
+  const int32_t t1 = (int32_t)((t0 + seg_len < T) ? t0 + seg_len : T);
   const DevPolicy P = pol[c0];
   const int W = W_T > 0 ? W_T : P.W;
   const int H = H_T > 0 ? H_T : P.H;
-  const int64_t wt0 = t0 >> 5;
-  const int64_t wend = (t1 + 31) >> 5;
-  int64_t nhalo = 0;
+  const int32_t wt0 = t0 >> 5;
+  const int32_t wend = (t1 + 31) >> 5;
+  int32_t nhalo = 0;
   if (s > 0) {
     nhalo = (W + H - 1 + 31) / 32;
     if (nhalo > wt0) nhalo = wt0;
   }
-  const int64_t w_first = wt0 - nhalo;
-  const int64_t nwords = wend - w_first;
+  const int32_t w_first = wt0 - nhalo;
+  const int32_t nwords = wend - w_first;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (warp == kConsumerWarps) {  // ---------------- producer warp ----------------
     if (lane == 0) {
       int st = 0;
       uint32_t ph = 0;
-      for (int64_t j = 0; j < nwords; ++j) {
+      for (int32_t j = 0; j < nwords; ++j) {
         if (j >= kStages) mbar_wait(&empty_bar[st], ph ^ 1u);
-        const int64_t w = w_first + j, p0 = w * 32;
+        const int32_t w = w_first + j, p0 = w * 32;
         st_mul[st] = digest_mul(w);
         st_warm[st] = (p0 >= W) ? 0u : ((W - p0) >= 32 ? ~0u : ((1u << (W - p0)) - 1u));
         st_tail[st] = tail_mask(p0, T);
@@ -336,14 +338,18 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
 #pragma unroll
   for (int k = 0; k < NB; ++k) {
     B.cnt_a[k] = 0; B.cnt_b[k] = 0; B.cnt_c[k] = 0; B.cnt_d[k] = 0; B.cnt_e[k] = 0;
+    B.cnt_f[k] = 0; B.cnt_g[k] = 0;
     B.qmin[k] = 0; B.dig[k] = 0; B.pqmin[k] = 0;
     bs[k][tid].qmax = 0; bs[k][tid].pqmax = 0; bs[k][tid].pdig = 0;
     bs[k][tid].apos = -1; bs[k][tid].wa = -1; bs[k][tid].dwa = 0; bs[k][tid].pre_dec_a = 0;
   }
   B.carry = hyp ? (1u << NB) - 1u : 0u;
   B.seen = 0; B.va = 0; B.last = 0;
-  uint32_t Eprev = 0, ev = 0;
+  uint32_t Eprev = 0, ev = 0, bbase = 0;
   unsigned long long qbase = 0;
+  constexpr bool bursts = BURST;                    // Sec. 6.3 Jaccard counters (f1)
+  const bool bkeep = plat.burst_min_keeps != 0;     // B_min > theta: no burst is hidden
+  const float xburst = plat.xburst;
   const bool want_dec = wk.dec != nullptr && valid;
   uint32_t* dec_row = want_dec ? wk.dec + wt0 * N + n : nullptr;  // + c * dec_cstride
   double pd[W_T > 1 ? W_T - 1 : 1];  // previous word's last W-1 samples, widened
@@ -352,11 +358,11 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
 
   int st = 0, pst = kStages - 1;
   uint32_t ph = 0;
-  for (int64_t j = 0; j < nwords; ++j) {
+  for (int32_t j = 0; j < nwords; ++j) {
     mbar_wait(&full_bar[st], ph);
     const float* cur = sm + st * kStageFloats + tid;
-    const int64_t w = w_first + j;
-    const int64_t p0 = w * 32;
+    const int32_t w = w_first + j;
+    const int32_t p0 = w * 32;
 
     // ---- per sample: Alg. 1 predicates + stretch flag, packed ----
     uint32_t incw = 0, decw = 0, smin = 0;
@@ -400,6 +406,13 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
       const uint64_t M = st_mul[st];
       const bool final_word = (w == wend - 1);
       ev += __popc(E & outm);
+      uint32_t bb = 0;  // bursts at max uncore: delivered x > theta
+      if constexpr (bursts) {
+#pragma unroll
+        for (int i = 0; i < 32; ++i) or_if_gt(bb, cur[i * kTraces], xburst, 1u << i);
+        bb &= outm;
+        bbase += __popc(bb);
+      }
       // Alg. 2 (l.9): the count of the H previous events, shared by the bundle
       uint32_t cnt[Window<H_T>::NBITS];
       Window<H_T>::count(E, Eprev, H, cnt);
@@ -450,6 +463,12 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
           bs[k][tid].pdig += (unsigned long long)pre_dec * M;
         } else if (want_dec && cfg[k] >= 0) {
           dec_row[(int64_t)cfg[k] * wk.dec_cstride] = Dout;
+        }
+        if constexpr (bursts) {  // kept unless the interval ran at a level whose capacity hides it
+          const uint32_t kept = bkeep ? bb : (bb & ~Lv[k]);
+          const uint32_t pb = bkeep ? 0u : (bb & pre_int[k]);
+          if constexpr (kPack) B.cnt_f[k] += (uint32_t)__popc(kept) | ((uint32_t)__popc(pb) << 16);
+          else { B.cnt_f[k] += __popc(kept); B.cnt_g[k] += __popc(pb); }
         }
         need_q |= (Lv[k] | pre_int[k]);
         B.carry = (B.carry & ~(1u << k)) | ((D >> 31) << k);
@@ -529,13 +548,15 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
         if (v & 2u) { cin = (v >> 2) & 1u; break; }
       }
     }
-    uint32_t hi, msr, mdec, mint, ch;
+    uint32_t hi, msr, mdec, mint, ch, bm, pb;
     if constexpr (kPack) {
       hi = B.cnt_a[k] & 0xFFFFu; msr = B.cnt_a[k] >> 16;
       mdec = B.cnt_b[k] & 0xFFFFu; mint = B.cnt_b[k] >> 16;
       ch = B.cnt_c[k];
+      bm = B.cnt_f[k] & 0xFFFFu; pb = B.cnt_f[k] >> 16;
     } else {
       hi = B.cnt_a[k]; msr = B.cnt_b[k]; mdec = B.cnt_c[k]; mint = B.cnt_d[k]; ch = B.cnt_e[k];
+      bm = B.cnt_f[k]; pb = B.cnt_g[k];
     }
     unsigned long long qmin = B.qmin[k], qmax = S.qmax, dig = B.dig[k];
     if (cin != hyp) {
@@ -544,9 +565,11 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
       if (hyp) {  // assumed min, truly max
         mint -= n_int; mdec -= n_dec;
         qmin -= B.pqmin[k]; qmax += S.pqmax; dig -= S.pdig;
+        bm += pb;
       } else {    // assumed max, truly min
         mint += n_int; mdec += n_dec;
         qmin += B.pqmin[k]; qmax -= S.pqmax; dig += S.pdig;
+        bm -= pb;
       }
       const uint32_t va = (B.va >> k) & 1u;
       if (seen) ch += (uint32_t)((int)(va != cin) - (int)(va != hyp));
@@ -554,8 +577,8 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
     if (want_dec) {  // deferred prefix decision words
       uint32_t* dec_out = wk.dec + (int64_t)c * wk.dec_cstride + n;
       const uint32_t fill = cin ? ~0u : 0u;
-      const int64_t wlast = seen ? wt0 + S.wa : wend;
-      for (int64_t w = wt0; w < wlast; ++w) dec_out[w * N] = fill & tail_mask(w * 32, T);
+      const int32_t wlast = seen ? wt0 + S.wa : wend;
+      for (int32_t w = wt0; w < wlast; ++w) dec_out[w * N] = fill & tail_mask(w * 32, T);
       if (seen) dec_out[(wt0 + S.wa) * N] = (S.dwa & ~S.pre_dec_a) | (fill & S.pre_dec_a);
     }
     // segment sums -> per-(config, trace) accumulators (exact integer atomics)
@@ -570,6 +593,10 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
     atomicAdd(acc + 7 * N, qmax);
     atomicAdd(acc + 8 * N, qbase);
     atomicAdd(acc + 9 * N, dig);
+    if constexpr (BURST) {  // (the burst accumulators stay zero otherwise)
+      atomicAdd(acc + 10 * N, (unsigned long long)bbase);
+      atomicAdd(acc + 11 * N, (unsigned long long)bm);
+    }
   }
   __threadfence();
   consumer_sync();
@@ -594,7 +621,8 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
         }
         magus_summary sm_out;
         finalize_summary(plat, T, (int64_t)a[0], (int64_t)a[1], (int64_t)a[2], (int64_t)a[3],
-                         (int64_t)a[4], (int64_t)a[5], a[6], a[7], a[8], a[9], &sm_out,
+                         (int64_t)a[4], (int64_t)a[5], a[6], a[7], a[8], a[9], (int64_t)a[10],
+                         (int64_t)a[11], &sm_out,
                          (wk.base && c == 0) ? wk.base + n : nullptr);
         if (wk.summary) wk.summary[(int64_t)c * N + n] = sm_out;
         tv[0] = (unsigned long long)sm_out.viol;
@@ -603,6 +631,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
         tv[7] = a[6] & 0xFFFFFFFFULL; tv[8] = a[6] >> 32;
         tv[9] = a[7] & 0xFFFFFFFFULL; tv[10] = a[7] >> 32;
         tv[11] = a[8] & 0xFFFFFFFFULL; tv[12] = a[8] >> 32;
+        tv[13] = a[10]; tv[14] = a[11];
       }
       if (wk.totals) {  // per-config fleet totals (exact integer sums)
 #pragma unroll
@@ -625,8 +654,9 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
         if (sh_last2) {
           __threadfence();
           uint64_t* out = wk.totals + (int64_t)c * MAGUS_TOT_WORDS;
-          if (tid < kTotAcc) {
-            out[1 + tid] = __ldcg(wk.tacc + (int64_t)c * kTotAcc + tid);
+          if (tid < kTotAcc) {  // accumulators 0..12 -> words 1..13; 13, 14 -> bursts
+            const int word = tid < 13 ? 1 + tid : MAGUS_TOT_BURST_BASE + (tid - 13);
+            out[word] = __ldcg(wk.tacc + (int64_t)c * kTotAcc + tid);
             wk.tacc[(int64_t)c * kTotAcc + tid] = 0ULL;
           }
           if (tid == 0) {
@@ -658,27 +688,32 @@ struct Pick {
   int smem;
 };
 
-template <int NB>
+template <int NB, bool BURST>
 Pick pick_nb(int32_t W, int32_t H) {
   if (H == 10) {
     switch (W) {
-      case 4: return {stream_kernel<4, 10, NB>, Stages<4>::smem};
-      case 6: return {stream_kernel<6, 10, NB>, Stages<6>::smem};
-      case 10: return {stream_kernel<10, 10, NB>, Stages<10>::smem};
-      case 16: return {stream_kernel<16, 10, NB>, Stages<16>::smem};
+      case 4: return {stream_kernel<4, 10, NB, BURST>, Stages<4>::smem};
+      case 6: return {stream_kernel<6, 10, NB, BURST>, Stages<6>::smem};
+      case 10: return {stream_kernel<10, 10, NB, BURST>, Stages<10>::smem};
+      case 16: return {stream_kernel<16, 10, NB, BURST>, Stages<16>::smem};
       default: break;
     }
-    if (W >= 2 && W <= 33) return {stream_kernel<0, 10, NB>, Stages<0>::smem};
+    if (W >= 2 && W <= 33) return {stream_kernel<0, 10, NB, BURST>, Stages<0>::smem};
   }
-  if (W >= 2 && W <= 33 && H >= 1 && H <= 32) return {stream_kernel<0, 0, NB>, Stages<0>::smem};
+  if (W >= 2 && W <= 33 && H >= 1 && H <= 32) return {stream_kernel<0, 0, NB, BURST>, Stages<0>::smem};
   return {nullptr, 0};
 }
 
-Pick pick(int32_t W, int32_t H, int32_t NB) {
-  switch (NB) {
-    case 1: return pick_nb<1>(W, H);
-    case 2: return pick_nb<2>(W, H);
-    case 4: return pick_nb<4>(W, H);
+// The Sec. 6.3 burst counters are a compile-time flag so that the default
+// path carries none of their registers.
+Pick pick(int32_t W, int32_t H, int32_t NB, bool burst = false) {
+  switch (NB * 2 + (burst ? 1 : 0)) {
+    case 2: return pick_nb<1, false>(W, H);
+    case 3: return pick_nb<1, true>(W, H);
+    case 4: return pick_nb<2, false>(W, H);
+    case 5: return pick_nb<2, true>(W, H);
+    case 8: return pick_nb<4, false>(W, H);
+    case 9: return pick_nb<4, true>(W, H);
     default: return {nullptr, 0};
   }
 }
@@ -702,7 +737,7 @@ int launch_stream(cudaStream_t st, const void* tmap, int64_t N, int64_t T,
                   const DevPolicy* pol_dev, const int32_t* bundles_dev, int32_t nbund, int32_t NB,
                   int32_t W, int32_t H, const DevPlatform& plat, int64_t nseg, int64_t seg_len,
                   const StreamWork& wk, int* grid_out) {
-  Pick p = pick(W, H, NB);
+  Pick p = pick(W, H, NB, plat.burst_on != 0);
   if (!p.f) return -1;
   cudaFuncSetAttribute((const void*)p.f, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem);
   const int32_t ngroups = (int32_t)((N + kTraces - 1) / kTraces);

@@ -39,20 +39,26 @@ struct DevPlatform {
   double invB24_min, invB24_max;
   // finalisation (fp64, fixed order)
   double dt, cQ, P_max, P_min, e_sw, t_sw, bound;
+  // Sec. 6.3 bursts: burst(t, l) <=> x_t > theta and B_l > theta
+  double burst_mbs, Bmin, Bmax;  // literal form (reference kernel)
+  float xburst;                  // x > xburst <=> (double)x > theta
+  int32_t burst_on;              // theta > 0 and B_max > theta
+  int32_t burst_min_keeps;       // B_min > theta: the level never hides a burst
+  int32_t pad_;
 };
 
 // Work/scratch block of the fused stream kernel (kernels_stream.cu).  The
 // counters and accumulators are zero at allocation and self-cleaning (the
 // last user of each resets it); the segment status words are tagged with a
 // per-replay epoch, so nothing needs a memset between replays.
-constexpr int kAccFields = 10;  // ev hi msr ch mdec mint qmin qmax qbase dig
+constexpr int kAccFields = 12;  // ev hi msr ch mdec mint qmin qmax qbase dig bbase bmagus
 struct StreamWork {
   uint32_t* ticket;              // [1] launch-order work ticket
   uint32_t* done;                // [1] finished CTAs of the launch
   uint32_t* status;              // [C][nseg][N] epoch<<3 | last_min<<2 | seen<<1 | 1
   unsigned long long* acc;       // [C][kAccFields][N] segment sums
   uint32_t* arrive;              // [C][ngroups] finished segments
-  unsigned long long* tacc;      // [C][13] totals under construction
+  unsigned long long* tacc;      // [C][kTotAccWords] totals under construction
   uint32_t* tarrive;             // [C] finished groups
   uint32_t epoch;
   magus_summary* summary;        // [C][N] or NULL
@@ -70,6 +76,8 @@ DevPlatform make_dev_platform(const magus_platform& p);
 double invert_inc(double L, double tau_inc);
 double invert_dec(double L, double tau_dec);
 float stretch_threshold(double invB);
+float above_threshold(double theta);  // largest float f with !((double)f > theta)
+constexpr int kTotAccWords = 15;      // totals words 1..13 + the two burst sums
 
 // Launchers (each returns the number of kernels launched, or -1 on error).
 

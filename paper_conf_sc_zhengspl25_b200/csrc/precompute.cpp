@@ -72,6 +72,24 @@ float stretch_threshold(double invB) {
   return f;
 }
 
+float above_threshold(double theta) {
+  // largest float f with !((double)f > theta); -inf when even -FLT_MAX exceeds it
+  if (!(theta < (double)3.4028234663852886e38)) return INFINITY;
+  int64_t lo = -(int64_t)0x7F800000, hi = 0x7F800000;  // ordered float keys: -inf .. +inf
+  auto val = [](int64_t k) {
+    uint32_t b = k >= 0 ? (uint32_t)k : ((uint32_t)(-k) | 0x80000000u);
+    float f;
+    std::memcpy(&f, &b, 4);
+    return f;
+  };
+  if ((double)val(lo) > theta) return -INFINITY;
+  while (hi - lo > 1) {
+    const int64_t mid = lo + (hi - lo) / 2;
+    if (!((double)val(mid) > theta)) lo = mid; else hi = mid;
+  }
+  return val(lo);
+}
+
 bool validate_policy(const magus_policy& p, char* msg, size_t n) {
   if (p.window < 2) { std::snprintf(msg, n, "window %d < 2", p.window); return false; }
   if (p.history < 1 || p.history > 64) {
@@ -96,7 +114,7 @@ bool validate_platform(const magus_platform& p, char* msg, size_t n) {
     return false;
   }
   const double v[] = {p.dt_s, p.bw_max_mbs, p.beta, p.p_other_w, p.p_unc_min_w, p.p_unc_max_w,
-                      p.e_switch_j, p.t_switch_s, p.slowdown_bound};
+                      p.e_switch_j, p.t_switch_s, p.slowdown_bound, p.burst_mbs};
   for (double d : v)
     if (!std::isfinite(d)) { std::snprintf(msg, n, "platform values must be finite"); return false; }
   if (!(p.dt_s > 0.0) || !(p.bw_max_mbs > 0.0)) {
@@ -151,6 +169,12 @@ DevPlatform make_dev_platform(const magus_platform& p) {
   d.e_sw = p.e_switch_j;
   d.t_sw = p.t_switch_s;
   d.bound = p.slowdown_bound;
+  d.burst_mbs = p.burst_mbs;
+  d.Bmin = Bmin;
+  d.Bmax = Bmax;
+  d.xburst = above_threshold(p.burst_mbs);
+  d.burst_on = (p.burst_mbs > 0.0 && Bmax > p.burst_mbs) ? 1 : 0;
+  d.burst_min_keeps = (Bmin > p.burst_mbs) ? 1 : 0;
   return d;
 }
 

@@ -75,16 +75,16 @@ def test_null_context_is_rejected():
 def test_ptxas_report_has_no_spills_on_the_hot_kernel():
     log = open(os.path.join(ROOT, "paper_conf_sc_zhengspl25_b200", "build", "ptxas.log")).read()
     blocks = re.split(r"Compiling entry function", log)
-    hot = [b for b in blocks if "stream_kernelILi10ELi10E" in b]
+    hot = [b for b in blocks if "stream_kernelILi10ELi10ELi1ELb0E" in b]
     assert hot, "stream_kernel<10,10> missing from the build"
     assert "0 bytes spill stores" in hot[0]
 
 
 def test_binding_structs_match_header_sizes():
     import paper_conf_sc_zhengspl25_b200 as m
-    assert ctypes.sizeof(m.Policy) == 40 and ctypes.sizeof(m.Platform) == 80
-    assert m.SUMMARY_DT.itemsize == 104 and m.BASE_DT.itemsize == 32
-    assert np.dtype(np.uint64).itemsize * m.TOT_WORDS == 128
+    assert ctypes.sizeof(m.Policy) == 40 and ctypes.sizeof(m.Platform) == 88
+    assert m.SUMMARY_DT.itemsize == 120 and m.BASE_DT.itemsize == 32
+    assert np.dtype(np.uint64).itemsize * m.TOT_WORDS == 144
 
 
 def _nextafter(x, d):
