@@ -73,7 +73,15 @@ typedef struct {
   double  tau_dec;   /* Alg. 1: d <  tau_dec -> -1. SIGNED: paper "500" is
                         read as -500 (reading R1).                 */
   double  t_hi;      /* Alg. 2: s/H >= t_hi -> high-frequency. Paper 0.4.    */
+  int32_t variant;   /* 0 = the paper's MAGUS.  NEXT rows:
+                        MAGUS_VARIANT_CLOSED_LOOP: Alg. 1 observes delivered
+                        throughput min(x_t, B(l_t)) instead of demand (f3);
+                        MAGUS_VARIANT_GRADUAL: +-step ratio per event instead
+                        of the jump to max/min (f4, the contrast of P@35554).
+                        Non-zero variants run in the per-sample kernel.      */
+  int32_t step;      /* ratio step of MAGUS_VARIANT_GRADUAL (>= 1), else 0   */
 } magus_policy;
+enum { MAGUS_VARIANT_CLOSED_LOOP = 1, MAGUS_VARIANT_GRADUAL = 2 };
 
 /* Platform + accounting model M (an assumption).
  * Validation: 1 <= ratio_min < ratio_max <= 127; dt_s > 0; bw_max_mbs > 0;
@@ -221,6 +229,15 @@ magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t n_traces,
                           const magus_policy* params, int32_t n_params,
                           magus_summary* out_summary, magus_base* out_base,
                           uint32_t* out_decisions, uint64_t* out_totals);
+
+/* Per-interval decisions as uncore ratios (needed for multi-level variants):
+ * out_levels DEVICE uint8 [n_params][n_steps][n_traces], level[c][t][n] =
+ * dec[t] of trace n under config c.  Runs the per-sample kernel; other
+ * outputs as in magus_replay.  Asynchronous. */
+magus_status magus_replay_levels(magus_ctx ctx, const float* traces, int64_t n_traces,
+                                 int64_t n_steps, int64_t ld, const magus_policy* params,
+                                 int32_t n_params, uint8_t* out_levels,
+                                 magus_summary* out_summary, uint64_t* out_totals);
 
 /* End-to-end variant: every pointer is HOST memory (pinned or pageable).
  * Stages traces host->device through context-owned buffers, runs

@@ -23,7 +23,8 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "liboracle.so")
 
 POLICY_DT = np.dtype([("W", "<i4"), ("H", "<i4"), ("L", "<f8"), ("tau_inc", "<f8"),
-                      ("tau_dec", "<f8"), ("t_hi", "<f8")], align=True)
+                      ("tau_dec", "<f8"), ("t_hi", "<f8"), ("variant", "<i4"), ("step", "<i4")],
+                     align=True)
 PLATFORM_DT = np.dtype([("r_min", "<i4"), ("r_max", "<i4"), ("dt", "<f8"), ("bw_max", "<f8"),
                         ("beta", "<f8"), ("p_other", "<f8"), ("p_unc_min", "<f8"),
                         ("p_unc_max", "<f8"), ("e_sw", "<f8"), ("t_sw", "<f8"),
@@ -76,13 +77,16 @@ def _load():
 # Paper parameters (restated here, independently of the product presets).
 # ---------------------------------------------------------------------------
 
-def policy(W=10, H=10, L=None, tau_inc=200.0, tau_dec=-500.0, t_hi=0.4) -> np.ndarray:
+def policy(W=10, H=10, L=None, tau_inc=200.0, tau_dec=-500.0, t_hi=0.4, variant=0, step=None) -> np.ndarray:
     """One config.  Defaults: P@25197 (200 / "500" read as -500 / 0.4), H = 10
-    (P@24182), W = 10 and L = W (readings R4/R5)."""
+    (P@24182), W = 10 and L = W (readings R4/R5).  variant: 0 the
+    paper's MAGUS; 1 closed loop (NEXT f3); 2 gradual +-step rule (NEXT f4)."""
     p = np.zeros(1, dtype=POLICY_DT)
     p["W"], p["H"] = W, H
     p["L"] = float(W if L is None else L)
     p["tau_inc"], p["tau_dec"], p["t_hi"] = tau_inc, tau_dec, t_hi
+    p["variant"] = variant
+    p["step"] = (1 if variant & 2 else 0) if step is None else step
     return p
 
 

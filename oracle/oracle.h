@@ -19,6 +19,8 @@ typedef struct {
   double tau_inc;   /* inc_threshold                           */
   double tau_dec;   /* dec_threshold (signed)                  */
   double t_hi;      /* high_freq_threshold                     */
+  int32_t variant;  /* 0 paper; 1 closed loop (f3); 2 gradual step (f4) */
+  int32_t step;     /* ratio step of the gradual variant       */
 } or_policy;
 
 typedef struct {

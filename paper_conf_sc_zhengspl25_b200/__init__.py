@@ -34,7 +34,8 @@ TOT_NAMES = ["n_traces", "n_viol", "events", "hi_rounds", "msr_writes", "changes
 
 class Policy(ctypes.Structure):
     _fields_ = [("window", ctypes.c_int32), ("history", ctypes.c_int32), ("deriv_len", ctypes.c_double),
-                ("tau_inc", ctypes.c_double), ("tau_dec", ctypes.c_double), ("t_hi", ctypes.c_double)]
+                ("tau_inc", ctypes.c_double), ("tau_dec", ctypes.c_double), ("t_hi", ctypes.c_double),
+                ("variant", ctypes.c_int32), ("step", ctypes.c_int32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -97,6 +98,7 @@ _lib.magus_grid_sweep256.argtypes = [ctypes.POINTER(Policy)]
 _lib.magus_grid_fleet64.argtypes = [ctypes.POINTER(Policy)]
 _lib.magus_replay.argtypes = [_vp, _vp, _i64, _i64, _i64, ctypes.POINTER(Policy), _i32, _vp, _vp, _vp, _vp]
 _lib.magus_replay_host.argtypes = [_vp, _vp, _i64, _i64, _i64, ctypes.POINTER(Policy), _i32, _vp, _vp, _vp, _vp]
+_lib.magus_replay_levels.argtypes = [_vp, _vp, _i64, _i64, _i64, ctypes.POINTER(Policy), _i32, _vp, _vp, _vp]
 _lib.magus_totals_derive.argtypes = [_vp, _vp, ctypes.POINTER(Derived)]
 _lib.magus_sweep_best.argtypes = [_vp, _vp, _i32, ctypes.POINTER(_i32), ctypes.POINTER(Derived)]
 _lib.magus_gen_traces.argtypes = [_vp, _u64, _i64, _i64, _i64, _i64, _i32, _vp]
@@ -114,7 +116,8 @@ for _f in ("magus_init", "magus_destroy", "magus_set_stream", "magus_policy_pres
            "magus_grid_sweep256", "magus_grid_fleet64", "magus_replay", "magus_replay_host",
            "magus_totals_derive", "magus_sweep_best", "magus_gen_traces", "magus_set_option",
            "magus_get_stats", "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
-           "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host"):
+           "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host",
+           "magus_replay_levels"):
     getattr(_lib, _f).restype = ctypes.c_int
 
 EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_string", "magus_last_error",
@@ -122,7 +125,9 @@ EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_str
             "magus_grid_fleet64", "magus_replay", "magus_replay_host", "magus_totals_derive",
             "magus_sweep_best", "magus_gen_traces", "magus_set_option", "magus_get_stats",
             "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
-            "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host"]
+            "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host",
+            "magus_replay_levels"]
+VARIANT_CLOSED_LOOP, VARIANT_GRADUAL = 1, 2
 
 
 class MagusError(RuntimeError):
@@ -216,8 +221,9 @@ def pareto_front_host(totals, platform: Platform | None = None) -> np.ndarray:
     return on.astype(bool)
 
 
-def make_policy(W=10, H=10, L=None, tau_inc=200.0, tau_dec=-500.0, t_hi=0.4) -> Policy:
-    return Policy(W, H, float(W if L is None else L), tau_inc, tau_dec, t_hi)
+def make_policy(W=10, H=10, L=None, tau_inc=200.0, tau_dec=-500.0, t_hi=0.4, variant=0, step=None) -> Policy:
+    step = (1 if variant & VARIANT_GRADUAL else 0) if step is None else step
+    return Policy(W, H, float(W if L is None else L), tau_inc, tau_dec, t_hi, variant, step)
 
 
 def _policy_array(policies) -> tuple[ctypes.Array, int]:
@@ -337,6 +343,26 @@ class Context:
                                p(out.decisions), p(out.totals))
         self._check(st, "replay")
         return out
+
+    def replay_levels(self, traces, policies, n_traces: int | None = None, want_totals: bool = True):
+        """Per-interval uncore ratios (uint8 [C, T, N]) + summaries (+ totals):
+        the per-sample kernel, required for the multi-level f4 variant."""
+        torch = self._torch
+        assert traces.is_cuda and traces.dtype == torch.float32 and traces.stride(1) == 1
+        T, ld = traces.shape[0], traces.stride(0)
+        N = traces.shape[1] if n_traces is None else n_traces
+        arr, C = _policy_array(policies)
+        dev = traces.device
+        levels = torch.empty((C, T, N), dtype=torch.uint8, device=dev)
+        res = ReplayResult(summary=torch.empty((C, N, SUMMARY_DT.itemsize), dtype=torch.uint8, device=dev),
+                           base=None, decisions=None,
+                           totals=torch.empty((C, TOT_WORDS), dtype=torch.int64, device=dev) if want_totals else None,
+                           n_traces=N, n_configs=C)
+        st = _lib.magus_replay_levels(self._h, _vp(traces.data_ptr()), N, T, ld, arr, C, _vp(levels.data_ptr()),
+                                      _vp(res.summary.data_ptr()),
+                                      _vp(res.totals.data_ptr()) if want_totals else None)
+        self._check(st, "replay_levels")
+        return levels, res
 
     def replay_host(self, traces: np.ndarray, policies, n_traces: int | None = None, want_summary=True,
                     want_base=True, want_decisions=False, want_totals=True):

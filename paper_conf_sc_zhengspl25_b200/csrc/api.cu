@@ -311,6 +311,8 @@ magus_status magus_policy_preset(int32_t id, magus_policy* out) {
   p.deriv_len = 10.0;   // reading R4: L = W
   p.tau_dec = -500.0;   // P@25197 "500", signed per reading R1
   p.t_hi = 0.4;         // P@25197
+  p.variant = 0;        // the paper's MAGUS
+  p.step = 0;
   if (id == MAGUS_POLICY_PAPER_DEFAULT) p.tau_inc = 200.0;       // P@25197 (Sec. 3.3)
   else if (id == MAGUS_POLICY_PAPER_PARETO) p.tau_inc = 300.0;   // P@44170 (Sec. 6.4)
   else return MAGUS_ERR_INVALID_ARG;
@@ -357,6 +359,8 @@ magus_status magus_grid_sweep256(magus_policy out[256]) {
           p.tau_inc = kGridInc[iInc];
           p.tau_dec = kGridDec[iDec];
           p.t_hi = kGridHi[iHi];
+        p.variant = 0;
+        p.step = 0;
         }
   return MAGUS_OK;
 }
@@ -373,6 +377,8 @@ magus_status magus_grid_fleet64(magus_policy out[64]) {
         p.tau_inc = kGridInc[iInc];
         p.tau_dec = kGridDec[iDec];
         p.t_hi = kGridHi[iHi];
+        p.variant = 0;
+        p.step = 0;
       }
   return MAGUS_OK;
 }
@@ -478,19 +484,25 @@ magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value) {
   return fail(ctx, MAGUS_ERR_INVALID_ARG, "unknown option %d", key);
 }
 
-magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t N, int64_t T, int64_t ld,
-                          const magus_policy* params, int32_t C, magus_summary* out_summary,
-                          magus_base* out_base, uint32_t* out_decisions, uint64_t* out_totals) {
+static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, int64_t T,
+                                int64_t ld, const magus_policy* params, int32_t C,
+                                magus_summary* out_summary, magus_base* out_base,
+                                uint32_t* out_decisions, uint64_t* out_totals, uint8_t* out_levels) {
   if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
   magus_status st = validate_replay(ctx, traces, N, T, ld, params, C);
   if (st != MAGUS_OK) return st;
   DeviceGuard dg(ctx->device);
   cudaGetLastError();
 
-  // kernel choice
-  bool all_stream = true;
-  for (int32_t c = 0; c < C; ++c)
-    all_stream = all_stream && stream_supported(params[c].window, params[c].history);
+  // kernel choice: the stream kernel runs the paper's MAGUS (variant 0) with
+  // W <= 33, H <= 32 on TMA-addressable traces; everything else, and any
+  // per-interval level output, runs the per-sample kernel
+  bool all_stream = out_levels == nullptr, multi = false;
+  for (int32_t c = 0; c < C; ++c) {
+    all_stream = all_stream && params[c].variant == 0 &&
+                 stream_supported(params[c].window, params[c].history);
+    multi = multi || (params[c].variant & MAGUS_VARIANT_GRADUAL) != 0;
+  }
   const bool tma_ok = ((uintptr_t)traces % 16 == 0) && (ld % 4 == 0);
   int kernel = (int)ctx->opt_kernel;
   if (kernel == 0) kernel = (all_stream && tma_ok) ? 2 : 1;
@@ -546,8 +558,10 @@ magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t N, int64_t
     magus_base* base = out_base;
     if (!base && out_totals) base = (magus_base*)sp;
     if (ctx->opt_timing) CK(cudaEventRecord(ev0, ctx->stream));
-    int r = launch_reference(ctx->stream, traces, N, T, ld, dev_policies(ctx), C, ctx->dplat, summ,
-                             base, out_decisions);
+    int r = launch_reference(ctx->stream, traces, N, T, ld, dev_policies(ctx), C, ctx->dplat,
+                             ctx->plat.bw_max_mbs, ctx->plat.p_other_w + ctx->plat.p_unc_min_w,
+                             ctx->plat.p_unc_max_w - ctx->plat.p_unc_min_w, multi, summ, base,
+                             out_decisions, out_levels);
     if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "reference kernel launch");
     launched += r;
     ctx->last_grid = (N * C + 127) / 128;
@@ -614,6 +628,24 @@ magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t N, int64_t
   ctx->last_segments = nseg;
   ctx->last_kernel = kernel;
   return MAGUS_OK;
+}
+
+magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t N, int64_t T, int64_t ld,
+                          const magus_policy* params, int32_t C, magus_summary* out_summary,
+                          magus_base* out_base, uint32_t* out_decisions, uint64_t* out_totals) {
+  return replay_impl(ctx, traces, N, T, ld, params, C, out_summary, out_base, out_decisions,
+                     out_totals, nullptr);
+}
+
+magus_status magus_replay_levels(magus_ctx ctx, const float* traces, int64_t N, int64_t T,
+                                 int64_t ld, const magus_policy* params, int32_t C,
+                                 uint8_t* out_levels, magus_summary* out_summary,
+                                 uint64_t* out_totals) {
+  if (ctx && !out_levels) return fail(ctx, MAGUS_ERR_INVALID_ARG, "out_levels is NULL");
+  if (ctx && ctx->opt_kernel == 2)
+    return fail(ctx, MAGUS_ERR_UNSUPPORTED, "per-interval levels come from the per-sample kernel");
+  return replay_impl(ctx, traces, N, T, ld, params, C, out_summary, nullptr, nullptr, out_totals,
+                     out_levels);
 }
 
 magus_status magus_replay_host(magus_ctx ctx, const float* traces_host, int64_t N, int64_t T,

@@ -27,6 +27,7 @@ struct DevPolicy {
   double t_hi;
   // Alg. 2 inverted form: s >= k  (k = H+1: never)
   int32_t W, H, k, pad;
+  int32_t variant, step;  // NEXT f3/f4 (per-sample kernel only)
 };
 
 // Platform / model-M constants.
@@ -81,9 +82,12 @@ constexpr int kTotAccWords = 15;      // totals words 1..13 + the two burst sums
 
 // Launchers (each returns the number of kernels launched, or -1 on error).
 
+// Per-sample kernel (kernels_ref.cu); multi = per-level accounting (gradual
+// variant); out_levels optional uint8 [C][T][N].
 int launch_reference(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,
-                     const DevPolicy* pol_dev, int32_t C, const DevPlatform& plat,
-                     magus_summary* out_summary, magus_base* out_base, uint32_t* out_dec);
+                     const DevPolicy* pol_dev, int32_t C, const DevPlatform& plat, double bw_max,
+                     double p_lo, double p_span, bool multi, magus_summary* out_summary,
+                     magus_base* out_base, uint32_t* out_dec, uint8_t* out_levels);
 
 bool stream_supported(int32_t W, int32_t H);
 // Fused stream kernel over nbund bundles of NB configs (bundles_dev:

@@ -105,6 +105,18 @@ bool validate_policy(const magus_policy& p, char* msg, size_t n) {
     return false;
   }
   if (!(p.t_hi > 0.0)) { std::snprintf(msg, n, "t_hi %g not > 0", p.t_hi); return false; }
+  if (p.variant < 0 || p.variant > (MAGUS_VARIANT_CLOSED_LOOP | MAGUS_VARIANT_GRADUAL)) {
+    std::snprintf(msg, n, "unknown variant %d", p.variant);
+    return false;
+  }
+  if ((p.variant & MAGUS_VARIANT_GRADUAL) ? p.step < 1 : p.step != 0) {
+    std::snprintf(msg, n, "step %d: >= 1 for the gradual variant, else 0", p.step);
+    return false;
+  }
+  if ((p.variant & MAGUS_VARIANT_CLOSED_LOOP) && p.window > 128) {
+    std::snprintf(msg, n, "closed-loop variant needs window <= 128");
+    return false;
+  }
   return true;
 }
 
@@ -140,6 +152,8 @@ DevPolicy make_dev_policy(const magus_policy& p) {
   d.t_hi = p.t_hi;
   d.W = p.window;
   d.H = p.history;
+  d.variant = p.variant;
+  d.step = p.step;
   d.k = p.history + 1;
   for (int s = 0; s <= p.history; ++s)
     if ((double)s / (double)p.history >= p.t_hi) { d.k = s; break; }

@@ -82,7 +82,7 @@ def test_ptxas_report_has_no_spills_on_the_hot_kernel():
 
 def test_binding_structs_match_header_sizes():
     import paper_conf_sc_zhengspl25_b200 as m
-    assert ctypes.sizeof(m.Policy) == 40 and ctypes.sizeof(m.Platform) == 88
+    assert ctypes.sizeof(m.Policy) == 48 and ctypes.sizeof(m.Platform) == 88
     assert m.SUMMARY_DT.itemsize == 120 and m.BASE_DT.itemsize == 32
     assert np.dtype(np.uint64).itemsize * m.TOT_WORDS == 144
 
