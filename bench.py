@@ -153,7 +153,8 @@ def policies_for(grid):
 def oracle_policies(pols):
     import oracle
     return oracle.policies([dict(W=p.window, H=p.history, L=p.deriv_len, tau_inc=p.tau_inc,
-                                 tau_dec=p.tau_dec, t_hi=p.t_hi) for p in pols])
+                                 tau_dec=p.tau_dec, t_hi=p.t_hi, variant=p.variant, step=p.step)
+                            for p in pols])
 
 
 def run_reference(args):
@@ -213,6 +214,10 @@ def run_ours(args):
     if args.no_decisions:
         want_dec = False
     pols = policies_for(grid)
+    if args.variant:  # NEXT f3 / f4: closed loop / gradual step (per-sample kernel)
+        for p in pols:
+            p.variant = args.variant
+            p.step = args.step if args.variant & magus.VARIANT_GRADUAL else 0
     C = len(pols)
     seed = SEED_BASE + args.config
     plat = magus.platform_preset()
@@ -358,7 +363,8 @@ def run_ours(args):
                        "n_configs": C, "decisions_emitted": want_dec, "seed": hex(seed),
                        "l2": f"inputs {N * T * 4 / 1e9:.2f} GB per GPU > 126 MB L2 (no flush needed)",
                        "parallelism": f"traces sharded over {world} GPU(s); 1 NCCL all-reduce of int64 totals",
-                       "segments": st["last_segments"], "kernel": "stream" if st["last_kernel"] == 2 else "reference"},
+                       "segments": st["last_segments"], "kernel": "stream" if st["last_kernel"] == 2 else "reference",
+                       "variant": args.variant, "step": args.step if args.variant & 2 else 0},
             "roofline": roof,
             "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": int(st["launches_total"]), "clocks": clk,
@@ -392,6 +398,8 @@ def main():
     ap.add_argument("--waves", type=int, default=0, help="MAGUS_OPT_WAVES (0 = library default)")
     ap.add_argument("--segments", type=int, default=0, help="MAGUS_OPT_SEGMENTS (0 = auto)")
     ap.add_argument("--bundle", type=int, default=0, help="MAGUS_OPT_BUNDLE (0 = auto, 1, 2, 4)")
+    ap.add_argument("--variant", type=int, default=0, help="NEXT f3 (1 closed loop) / f4 (2 gradual)")
+    ap.add_argument("--step", type=int, default=1, help="ratio step of the gradual variant")
     ap.add_argument("--burst", type=float, default=0.0,
                     help="NEXT f1: Sec. 6.3 burst threshold (MB/s); > 0 enables the Jaccard counters")
     ap.add_argument("--no-e2e", action="store_true")

@@ -560,7 +560,8 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     if (ctx->opt_timing) CK(cudaEventRecord(ev0, ctx->stream));
     int r = launch_reference(ctx->stream, traces, N, T, ld, dev_policies(ctx), C, ctx->dplat,
                              ctx->plat.bw_max_mbs, ctx->plat.p_other_w + ctx->plat.p_unc_min_w,
-                             ctx->plat.p_unc_max_w - ctx->plat.p_unc_min_w, multi, summ, base,
+                             ctx->plat.p_unc_max_w - ctx->plat.p_unc_min_w, multi,
+                             /*literal=*/ctx->opt_kernel == 1, summ, base,
                              out_decisions, out_levels);
     if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "reference kernel launch");
     launched += r;

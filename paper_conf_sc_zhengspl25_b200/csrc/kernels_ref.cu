@@ -27,7 +27,11 @@ __device__ __forceinline__ double capacity(const DevPlatform& p, double bw_max, 
   return (bw_max * (double)l) / (double)p.r_max;
 }
 
-template <bool MULTI>
+// LITERAL: Alg. 1/2 with the printed fp64 divisions (the parity baseline of
+// the stream kernel); otherwise the exact host-inverted thresholds of
+// precompute.cpp (delta > d_inc, s >= k), which shortens the dependent chain
+// of the sequential variants by two fp64 divisions per round.
+template <bool MULTI, bool LITERAL>
 __global__ void __launch_bounds__(128)
 ref_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
            const DevPolicy* __restrict__ pol, int32_t C, DevPlatform plat, double bw_max,
@@ -71,13 +75,26 @@ ref_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
     for (int i = 0; i < nlev; ++i) { nl[i] = 0; ql[i] = 0; }
   }
 
+  // The scan is sequential, but its inputs are not: each 32-step chunk of
+  // samples and of their Alg. 1 lags is loaded up front (64 independent
+  // coalesced loads), so the dependent chain never waits on memory.
+  // (staged through this thread's columns of a shared-memory tile)
+  __shared__ float s_x[32][128], s_l[32][128];
   for (int64_t t = 0; t < T; ++t) {
-    const float xt = x[t * ld + n];
+    const int j = (int)(t & 31);
+    if (j == 0) {
+#pragma unroll 8
+      for (int i = 0; i < 32; ++i) {
+        const int64_t ti = t + i, tli = ti - P.W + 1;
+        s_x[i][threadIdx.x] = ti < T ? x[ti * ld + n] : 0.0f;
+        s_l[i][threadIdx.x] = (ti < T && tli >= 0) ? x[tli * ld + n] : 0.0f;
+      }
+    }
+    const float xt = s_x[j][threadIdx.x], xl = s_l[j][threadIdx.x];
     const int leff = prev;       // model M / closed loop: interval t runs at dec[t-1] (R6)
     if (closed) ring[t & (kMaxLevels - 1)] = (uint8_t)leff;
     if (t >= P.W) {              // MDFS rounds start at t = W (reading R5)
       const int64_t tl = t - P.W + 1;
-      const float xl = x[tl * ld + n];
       double yt = (double)xt, yl = (double)xl;
       if (closed) {              // f3: delivered throughput min(x, B(level))
         const double Bt = s_B[leff - lmin], Bl = s_B[ring[tl & (kMaxLevels - 1)] - lmin];
@@ -86,11 +103,17 @@ ref_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
       }
       // Alg. 2: s = sum of the H logged events, f = s / n, f >= t_hi
       const int s = __popcll(hist);
-      const bool hi = ((double)s / (double)P.H) >= P.t_hi;
+      const bool hi = LITERAL ? ((double)s / (double)P.H) >= P.t_hi : s >= P.k;
       if (hi) { lvl = lmax; ++msr; ++hi_rounds; }
       // Alg. 1: d = (ls[n] - ls[0]) / L
-      const double d = (yt - yl) / P.L;
-      const int p = d > P.tau_inc ? 1 : (d < P.tau_dec ? -1 : 0);
+      int p;
+      if (LITERAL) {
+        const double d = (yt - yl) / P.L;
+        p = d > P.tau_inc ? 1 : (d < P.tau_dec ? -1 : 0);
+      } else {
+        const double D = yt - yl;
+        p = D > P.d_inc ? 1 : (D < P.d_dec ? -1 : 0);
+      }
       if (p != 0) {
         ++events;
         if (!hi) {
@@ -152,16 +175,14 @@ ref_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
 
 int launch_reference(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,
                      const DevPolicy* pol_dev, int32_t C, const DevPlatform& plat, double bw_max,
-                     double p_lo, double p_span, bool multi, magus_summary* out_summary,
+                     double p_lo, double p_span, bool multi, bool literal, magus_summary* out_summary,
                      magus_base* out_base, uint32_t* out_dec, uint8_t* out_levels) {
   const int64_t total = N * C;
-  const int64_t blocks = (total + 127) / 128;
-  if (multi)
-    ref_kernel<true><<<(unsigned)blocks, 128, 0, s>>>(x, N, T, ld, pol_dev, C, plat, bw_max, p_lo, p_span,
-                                                      out_summary, out_base, out_dec, out_levels);
-  else
-    ref_kernel<false><<<(unsigned)blocks, 128, 0, s>>>(x, N, T, ld, pol_dev, C, plat, bw_max, p_lo,
-                                                       p_span, out_summary, out_base, out_dec, out_levels);
+  const unsigned blocks = (unsigned)((total + 127) / 128);
+  auto k = multi ? (literal ? ref_kernel<true, true> : ref_kernel<true, false>)
+                 : (literal ? ref_kernel<false, true> : ref_kernel<false, false>);
+  k<<<blocks, 128, 0, s>>>(x, N, T, ld, pol_dev, C, plat, bw_max, p_lo, p_span, out_summary, out_base,
+                           out_dec, out_levels);
   return cudaGetLastError() == cudaSuccess ? 1 : -1;
 }
 

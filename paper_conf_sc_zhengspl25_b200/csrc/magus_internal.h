@@ -86,7 +86,7 @@ constexpr int kTotAccWords = 15;      // totals words 1..13 + the two burst sums
 // variant); out_levels optional uint8 [C][T][N].
 int launch_reference(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,
                      const DevPolicy* pol_dev, int32_t C, const DevPlatform& plat, double bw_max,
-                     double p_lo, double p_span, bool multi, magus_summary* out_summary,
+                     double p_lo, double p_span, bool multi, bool literal, magus_summary* out_summary,
                      magus_base* out_base, uint32_t* out_dec, uint8_t* out_levels);
 
 bool stream_supported(int32_t W, int32_t H);
