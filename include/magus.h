@@ -239,6 +239,21 @@ magus_status magus_replay_levels(magus_ctx ctx, const float* traces, int64_t n_t
                                  int32_t n_params, uint8_t* out_levels,
                                  magus_summary* out_summary, uint64_t* out_totals);
 
+/* NEXT f2: offline-optimal schedules under model M.
+ * For every trace and every Lagrange weight lambda_j >= 0 (HOST array),
+ * the schedule dec[0..T-1] over the level set (full_grid = 0: {ratio_min,
+ * ratio_max}, MAGUS's decision space; 1: every ratio in between) that
+ * minimises  energy + lambda * time  of model M, by an exact DP in time order
+ * with deterministic tie-breaks (stay before move; lowest ratio first).
+ * out DEVICE double [n_traces][n_lambda][3] = {minimal cost, energy, time}
+ * of that schedule (energy/time summed along the path in time order).
+ * lambda = 0 gives the least energy any schedule reaches: a lower bound MAGUS
+ * cannot beat; max_j (cost_j - lambda_j * (1 + bound) * base_time) is the
+ * Lagrangian lower bound of the slowdown-constrained problem.  Asynchronous. */
+magus_status magus_offline_bound(magus_ctx ctx, const float* traces, int64_t n_traces,
+                                 int64_t n_steps, int64_t ld, const double* lambdas,
+                                 int32_t n_lambda, int32_t full_grid, double* out);
+
 /* End-to-end variant: every pointer is HOST memory (pinned or pageable).
  * Stages traces host->device through context-owned buffers, runs
  * magus_replay, copies the requested outputs back.  Synchronises. */

@@ -62,6 +62,8 @@ def _load():
     lib.oracle_totals.argtypes = [vp, vp, i64, i64, vp, vp, vp]
     lib.oracle_energy_sum.restype = ctypes.c_double
     lib.oracle_energy_sum.argtypes = [vp, i64]
+    lib.oracle_offline_bound.restype = ctypes.c_int
+    lib.oracle_offline_bound.argtypes = [vp, i64, vp, f64, i32, vp]
     lib.oracle_sweep_best.restype = ctypes.c_int
     lib.oracle_sweep_best.argtypes = [vp, vp, i32, vp]
     for n in ("summary", "policy", "platform"):
@@ -184,6 +186,19 @@ def totals(summary_row: np.ndarray, base: np.ndarray, T: int, plat=None):
     if rc != 0:
         raise ValueError("oracle_totals rejected its arguments")
     return w, f
+
+
+def offline_bound(x, lam: float, plat=None, full_grid: bool = False) -> np.ndarray:
+    """NEXT f2 DP for one trace: {cost, energy, time} of the schedule that
+    minimises energy + lam * time under model M (magus_oracle.cpp)."""
+    x = np.ascontiguousarray(x, dtype=np.float32).reshape(-1)
+    plat = platform() if plat is None else np.ascontiguousarray(plat, dtype=PLATFORM_DT)
+    out = np.zeros(3, np.float64)
+    rc = _load().oracle_offline_bound(x.ctypes.data, len(x), plat.ctypes.data, float(lam), int(full_grid),
+                                      out.ctypes.data)
+    if rc != 0:
+        raise ValueError("oracle_offline_bound rejected its arguments")
+    return out
 
 
 def pareto_front(energy, time) -> np.ndarray:

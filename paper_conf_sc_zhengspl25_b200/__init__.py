@@ -99,6 +99,7 @@ _lib.magus_grid_fleet64.argtypes = [ctypes.POINTER(Policy)]
 _lib.magus_replay.argtypes = [_vp, _vp, _i64, _i64, _i64, ctypes.POINTER(Policy), _i32, _vp, _vp, _vp, _vp]
 _lib.magus_replay_host.argtypes = [_vp, _vp, _i64, _i64, _i64, ctypes.POINTER(Policy), _i32, _vp, _vp, _vp, _vp]
 _lib.magus_replay_levels.argtypes = [_vp, _vp, _i64, _i64, _i64, ctypes.POINTER(Policy), _i32, _vp, _vp, _vp]
+_lib.magus_offline_bound.argtypes = [_vp, _vp, _i64, _i64, _i64, _vp, _i32, _i32, _vp]
 _lib.magus_totals_derive.argtypes = [_vp, _vp, ctypes.POINTER(Derived)]
 _lib.magus_sweep_best.argtypes = [_vp, _vp, _i32, ctypes.POINTER(_i32), ctypes.POINTER(Derived)]
 _lib.magus_gen_traces.argtypes = [_vp, _u64, _i64, _i64, _i64, _i64, _i32, _vp]
@@ -117,7 +118,7 @@ for _f in ("magus_init", "magus_destroy", "magus_set_stream", "magus_policy_pres
            "magus_totals_derive", "magus_sweep_best", "magus_gen_traces", "magus_set_option",
            "magus_get_stats", "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
            "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host",
-           "magus_replay_levels"):
+           "magus_replay_levels", "magus_offline_bound"):
     getattr(_lib, _f).restype = ctypes.c_int
 
 EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_string", "magus_last_error",
@@ -126,7 +127,7 @@ EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_str
             "magus_sweep_best", "magus_gen_traces", "magus_set_option", "magus_get_stats",
             "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
             "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host",
-            "magus_replay_levels"]
+            "magus_replay_levels", "magus_offline_bound"]
 VARIANT_CLOSED_LOOP, VARIANT_GRADUAL = 1, 2
 
 
@@ -363,6 +364,20 @@ class Context:
                                       _vp(res.totals.data_ptr()) if want_totals else None)
         self._check(st, "replay_levels")
         return levels, res
+
+    def offline_bound(self, traces, lambdas, full_grid: bool = False, n_traces: int | None = None):
+        """NEXT f2: float64 tensor [N, len(lambdas), 3] = {cost, energy, time}
+        of the schedule minimising energy + lambda * time (magus_offline_bound)."""
+        torch = self._torch
+        assert traces.is_cuda and traces.dtype == torch.float32 and traces.stride(1) == 1
+        T, ld = traces.shape[0], traces.stride(0)
+        N = traces.shape[1] if n_traces is None else n_traces
+        lam = np.ascontiguousarray(lambdas, dtype=np.float64)
+        out = torch.empty((N, len(lam), 3), dtype=torch.float64, device=traces.device)
+        st = _lib.magus_offline_bound(self._h, _vp(traces.data_ptr()), N, T, ld, _vp(lam.ctypes.data), len(lam),
+                                      int(full_grid), _vp(out.data_ptr()))
+        self._check(st, "offline_bound")
+        return out
 
     def replay_host(self, traces: np.ndarray, policies, n_traces: int | None = None, want_summary=True,
                     want_base=True, want_decisions=False, want_totals=True):

@@ -49,6 +49,8 @@ struct magus_ctx_s {
   int64_t opt_bundle = 0;           // 0 auto, else force NB in {1, 2, 4}
   int64_t uploaded_bundle_opt = -1;
   // e2e staging (device)
+  void* lam_dev = nullptr;  // NEXT f2 lambda grid
+  size_t lam_bytes = 0;
   void* stage_dev = nullptr;
   size_t stage_bytes = 0;
   // stats
@@ -439,6 +441,7 @@ magus_status magus_destroy(magus_ctx ctx) {
     if (ctx->pol_dev) cudaFree(ctx->pol_dev);
     if (ctx->pol_host) cudaFreeHost(ctx->pol_host);
     if (ctx->best_pinned) cudaFreeHost(ctx->best_pinned);
+    if (ctx->lam_dev) cudaFree(ctx->lam_dev);
     if (ctx->stage_dev) cudaFree(ctx->stage_dev);
     if (ctx->pol_copied) cudaEventDestroy(ctx->pol_copied);
     for (auto& pr : ctx->pending) {
@@ -647,6 +650,36 @@ magus_status magus_replay_levels(magus_ctx ctx, const float* traces, int64_t N, 
     return fail(ctx, MAGUS_ERR_UNSUPPORTED, "per-interval levels come from the per-sample kernel");
   return replay_impl(ctx, traces, N, T, ld, params, C, out_summary, nullptr, nullptr, out_totals,
                      out_levels);
+}
+
+magus_status magus_offline_bound(magus_ctx ctx, const float* traces, int64_t N, int64_t T,
+                                 int64_t ld, const double* lambdas, int32_t nl, int32_t full_grid,
+                                 double* out) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  if (!traces || !out || !lambdas || nl < 1 || N < 1 || T < 1 || T > kMaxSteps || ld < N)
+    return fail(ctx, MAGUS_ERR_INVALID_ARG, "bad offline_bound arguments");
+  for (int32_t j = 0; j < nl; ++j)
+    if (!(lambdas[j] >= 0.0) || !std::isfinite(lambdas[j]))
+      return fail(ctx, MAGUS_ERR_INVALID_ARG, "lambda[%d] must be finite and >= 0", j);
+  if (full_grid && ctx->plat.ratio_max - ctx->plat.ratio_min + 1 > 32)
+    return fail(ctx, MAGUS_ERR_UNSUPPORTED, "the full grid supports at most 32 levels");
+  DeviceGuard dg(ctx->device);
+  const size_t need = sizeof(double) * (size_t)nl;
+  if (need > ctx->lam_bytes) {
+    CK(cudaStreamSynchronize(ctx->stream));
+    if (ctx->lam_dev) cudaFree(ctx->lam_dev);
+    ctx->lam_dev = nullptr;
+    CK(cudaMalloc(&ctx->lam_dev, need));
+    ctx->lam_bytes = need;
+  }
+  // pageable source: returns once staged, so `lambdas` may be reused at once
+  CK(cudaMemcpyAsync(ctx->lam_dev, lambdas, need, cudaMemcpyHostToDevice, ctx->stream));
+  const int r = launch_bound(ctx->stream, traces, N, T, ld, (const double*)ctx->lam_dev, nl, full_grid != 0,
+                             ctx->dplat, ctx->plat.bw_max_mbs, ctx->plat.p_other_w + ctx->plat.p_unc_min_w,
+                             ctx->plat.p_unc_max_w - ctx->plat.p_unc_min_w, out);
+  if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "bound kernel launch");
+  ctx->launches += r;
+  return MAGUS_OK;
 }
 
 magus_status magus_replay_host(magus_ctx ctx, const float* traces_host, int64_t N, int64_t T,

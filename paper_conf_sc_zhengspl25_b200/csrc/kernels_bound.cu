@@ -1,0 +1,119 @@
+// kernels_bound.cu -- NEXT f2: offline-optimal schedules under model M.
+//
+// For each (trace, lambda) the DP over the level set finds the schedule
+// dec[0..T-1] minimising energy + lambda * time of model M:
+//   interval t runs at l_t = dec[t-1] (l_0 = r_max, reading R6);
+//   cost of interval t at level l: c = e + lambda * tau with
+//     tau = dt + cQ * q(x_t, l),  e = P_l * tau   (model M 4.2-4.3);
+//   a change dec[t-1] != dec[t-2] (t >= 2, model M counts changes from t = 1)
+//   costs e_sw + lambda * t_sw.
+// V_t(i) = c(t, i) + min(V_{t-1}(i), min_{i' != i} V_{t-1}(i') + switch);
+// ties: stay before move, lowest level index first.  Energy and time are
+// summed along the chosen path in time order.  One thread per (trace,
+// lambda); the level states live in registers (binary set) or local memory.
+#include "device_common.cuh"
+
+namespace magus {
+
+constexpr int kBoundThreads = 128;
+
+template <int MAXL>
+__global__ void __launch_bounds__(kBoundThreads)
+bound_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
+             const double* __restrict__ lambdas, int32_t nl, int32_t L, int32_t l0, int32_t lstep,
+             DevPlatform plat, double bw_max, double p_lo, double p_span, double* __restrict__ out) {
+  __shared__ double s_invB[32], s_P[32];
+  __shared__ float s_x[32][kBoundThreads];
+  for (int i = threadIdx.x; i < L; i += blockDim.x) {
+    const int l = l0 + i * lstep;
+    const double B = (bw_max * (double)l) / (double)plat.r_max;
+    s_invB[i] = 1.0 / B;
+    s_P[i] = p_lo + (p_span * (double)(l - plat.r_min)) / (double)(plat.r_max - plat.r_min);
+  }
+  __syncthreads();
+  const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const bool active = gid < N * nl;
+  const int32_t j = active ? (int32_t)(gid / N) : 0;
+  const int64_t n = active ? gid - (int64_t)j * N : 0;
+  const double lam = lambdas[j];
+  const double sw_c = plat.e_sw + lam * plat.t_sw;
+  const int imax = L - 1;  // the level set is ascending and ends at r_max
+
+  double V[MAXL], E[MAXL], Tm[MAXL];
+  for (int i = 0; i < L; ++i) { V[i] = INFINITY; E[i] = 0.0; Tm[i] = 0.0; }
+
+  for (int64_t t = 0; t < T; ++t) {
+    const int jj = (int)(t & 31);
+    if (jj == 0) {  // stage the next 32 samples of this trace (independent loads)
+      __syncwarp();
+#pragma unroll 8
+      for (int i = 0; i < 32; ++i)
+        s_x[i][threadIdx.x] = (active && t + i < T) ? x[(t + i) * ld + n] : 0.0f;
+      __syncwarp();
+    }
+    const float xt = s_x[jj][threadIdx.x];
+    if (t == 0) {
+      const double tau = plat.dt + plat.cQ * (double)q_literal(xt, s_invB[imax]);
+      const double e = s_P[imax] * tau;
+      V[imax] = e + lam * tau;
+      E[imax] = e;
+      Tm[imax] = tau;
+      continue;
+    }
+    // best and second best previous state (lowest index on ties)
+    int a1 = 0;
+    double m1 = V[0];
+    for (int i = 1; i < L; ++i)
+      if (V[i] < m1) { m1 = V[i]; a1 = i; }
+    int a2 = -1;
+    double m2 = INFINITY;
+    for (int i = 0; i < L; ++i)
+      if (i != a1 && (a2 < 0 || V[i] < m2)) { m2 = V[i]; a2 = i; }
+    const bool sw = t >= 2;
+    double nV[MAXL], nE[MAXL], nT[MAXL];
+    for (int i = 0; i < L; ++i) {
+      const int oi = (i == a1) ? a2 : a1;
+      const double other = (i == a1) ? m2 : m1;
+      const double move = sw ? other + sw_c : other;
+      double v, e0, t0;
+      if (oi < 0 || V[i] <= move) {
+        v = V[i]; e0 = E[i]; t0 = Tm[i];
+      } else {
+        v = move;
+        e0 = sw ? E[oi] + plat.e_sw : E[oi];
+        t0 = sw ? Tm[oi] + plat.t_sw : Tm[oi];
+      }
+      const double tau = plat.dt + plat.cQ * (double)q_literal(xt, s_invB[i]);
+      const double e = s_P[i] * tau;
+      nV[i] = v + (e + lam * tau);
+      nE[i] = e0 + e;
+      nT[i] = t0 + tau;
+    }
+    for (int i = 0; i < L; ++i) { V[i] = nV[i]; E[i] = nE[i]; Tm[i] = nT[i]; }
+  }
+  if (!active) return;
+  int b = 0;
+  for (int i = 1; i < L; ++i)
+    if (V[i] < V[b]) b = i;
+  double* o = out + ((int64_t)n * nl + j) * 3;
+  o[0] = V[b];
+  o[1] = E[b];
+  o[2] = Tm[b];
+}
+
+int launch_bound(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,
+                 const double* lambdas_dev, int32_t nl, bool full_grid, const DevPlatform& plat,
+                 double bw_max, double p_lo, double p_span, double* out) {
+  const int32_t L = full_grid ? plat.r_max - plat.r_min + 1 : 2;
+  const int32_t lstep = full_grid ? 1 : plat.r_max - plat.r_min;
+  const unsigned blocks = (unsigned)((N * nl + kBoundThreads - 1) / kBoundThreads);
+  if (L == 2)
+    bound_kernel<2><<<blocks, kBoundThreads, 0, s>>>(x, N, T, ld, lambdas_dev, nl, L, plat.r_min, lstep,
+                                                     plat, bw_max, p_lo, p_span, out);
+  else
+    bound_kernel<32><<<blocks, kBoundThreads, 0, s>>>(x, N, T, ld, lambdas_dev, nl, L, plat.r_min, lstep,
+                                                      plat, bw_max, p_lo, p_span, out);
+  return cudaGetLastError() == cudaSuccess ? 1 : -1;
+}
+
+}  // namespace magus

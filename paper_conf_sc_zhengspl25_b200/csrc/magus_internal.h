@@ -100,6 +100,11 @@ int launch_stream(cudaStream_t s, const void* tmap /* CUtensorMap, host copy */,
                   int64_t seg_len, const StreamWork& wk, int* grid_out);
 int stream_ctas_per_sm(int32_t W, int32_t H, int32_t NB);
 
+// NEXT f2 DP (kernels_bound.cu): out [N][nl][3] = {cost, energy, time}.
+int launch_bound(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,
+                 const double* lambdas_dev, int32_t nl, bool full_grid, const DevPlatform& plat,
+                 double bw_max, double p_lo, double p_span, double* out);
+
 int launch_totals(cudaStream_t s, const magus_summary* summary, const magus_base* base, int64_t N,
                   int64_t T, int32_t C, uint64_t* totals);
 
