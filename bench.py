@@ -125,7 +125,9 @@ def cpu_oracle_sample(cfg, T, pols_oracle, budget_s, kind, max_traces=None):
     import gen
     import oracle
     seed = SEED_BASE + cfg
-    probe_n = 2
+    # probe on a sample of the same shape class (time-major, ld = n): the
+    # oracle reads each trace with stride ld, so a tiny probe under-estimates
+    probe_n = 64 if not max_traces else min(64, max_traces)
     xs = gen.gen_traces(seed, probe_n, T, kind=kind)
     t = time.perf_counter()
     oracle.replay(xs, pols_oracle)
@@ -133,6 +135,7 @@ def cpu_oracle_sample(cfg, T, pols_oracle, budget_s, kind, max_traces=None):
     n = max(1, int(budget_s / max(per_trace, 1e-9)))
     if max_traces:
         n = min(n, max_traces)
+    n = min(n, 1024)  # keeps ld (the oracle's stride) in the probed regime
     xs = gen.gen_traces(seed, n, T, kind=kind)
     t = time.perf_counter()
     ref = oracle.replay(xs, pols_oracle)
@@ -327,7 +330,7 @@ def run_ours(args):
         pol_o = oracle_policies(pols)
         if C > 16:
             pol_o = pol_o[:16]
-        v, n_s, dt_s, ref = cpu_oracle_sample(args.config, T, pol_o, args.cpu_budget, kind)
+        v, n_s, dt_s, ref = cpu_oracle_sample(args.config, T, pol_o, args.cpu_budget, kind, max_traces=N)
         cpu = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
                "sample": f"first {n_s} traces x {T} intervals x {len(pol_o)} config(s) of the same workload "
                          f"({dt_s:.1f} s single-threaded)"}
@@ -385,10 +388,70 @@ def run_ours(args):
     return 0
 
 
+def run_bound(args):
+    """NEXT f2: offline-optimal schedules (DP) on the workload, n_lambda weights.
+    Unit: trace-sample x lambda.  ALU-bound on the fp64 pipe: ~12 fp64 ops per
+    (trace-sample, lambda, level) (stretch, tau, energy, cost, 3 path sums);
+    peak = 148 SMs x 64 fp64 lanes x clock (B200 fp64 rate, half of fp32)."""
+    import torch
+
+    import oracle
+    import paper_conf_sc_zhengspl25_b200 as magus
+    N, T, _, kind, _, desc = WORKLOADS[args.config]
+    if args.n_traces:
+        N = args.n_traces
+    if args.n_steps:
+        T = args.n_steps
+    lams = [0.0] + [10.0 * 4 ** i for i in range(args.bound - 1)]
+    L = (22 - 8 + 1) if args.full_grid else 2
+    ctx = magus.Context(device=0)
+    x = ctx.gen_traces(SEED_BASE + args.config, N, T, kind=kind)
+    for _ in range(args.warmup):
+        out = ctx.offline_bound(x, lams, full_grid=args.full_grid)
+    torch.cuda.synchronize()
+    clocks = ClockSampler(0)
+    clocks.start()
+    time.sleep(0.2)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    clocks.mark()
+    e0.record()
+    for _ in range(args.steps):
+        out = ctx.offline_bound(x, lams, full_grid=args.full_grid)
+        out[0, 0, 0].item()  # device->host read of the result
+    e1.record()
+    torch.cuda.synchronize()
+    clocks.mark()
+    clocks.stop()
+    ms = e0.elapsed_time(e1) / args.steps
+    units = N * T * len(lams)
+    value = units / (ms * 1e-3)
+    clk = clocks.summary()
+    sm_mhz = clk.get("sm_max_mhz") or 1965.0
+    peak = 148 * 64 * sm_mhz * 1e6 / 1e9
+    ach = 12.0 * L * units / (ms * 1e-3) / 1e9
+    # parity of a few traces against the oracle's DP (untimed)
+    got = out.cpu().numpy()
+    xs = x[:, :4].cpu().numpy()
+    parity = all(np.array_equal(got[n, j], oracle.offline_bound(xs[:, n], lam, full_grid=args.full_grid))
+                 for n in range(4) for j, lam in enumerate(lams))
+    line = {"metric": "trace-samples x lambdas/sec (NEXT f2 offline-optimal DP)", "value": value,
+            "unit": "trace-samples*lambdas/s", "n_gpus": 1, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": desc, "n_traces": N, "n_steps": T, "lambdas": lams,
+                                             "levels": L},
+            "roofline": {"bound": "alu", "achieved": ach, "peak": peak, "unit": "Gop/s (fp64)",
+                         "frac": ach / peak, "traffic": None, "alg_ops_per_unit_level": 12,
+                         "peak_source": f"148 SMs x 64 fp64 lanes x {sm_mhz:.0f} MHz"},
+            "gpu_launches": int(ctx.stats()["launches_total"]), "clocks": clk, "parity_sample_ok": bool(parity)}
+    print(json.dumps(line), flush=True)
+    ctx.close()
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--steps", type=int, default=1000)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", type=int, default=2, choices=sorted(WORKLOADS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -398,6 +461,9 @@ def main():
     ap.add_argument("--waves", type=int, default=0, help="MAGUS_OPT_WAVES (0 = library default)")
     ap.add_argument("--segments", type=int, default=0, help="MAGUS_OPT_SEGMENTS (0 = auto)")
     ap.add_argument("--bundle", type=int, default=0, help="MAGUS_OPT_BUNDLE (0 = auto, 1, 2, 4)")
+    ap.add_argument("--bound", type=int, default=0,
+                    help="NEXT f2: time magus_offline_bound with this many lambdas instead of the replay")
+    ap.add_argument("--full-grid", action="store_true", help="f2 over every ratio, not {min, max}")
     ap.add_argument("--variant", type=int, default=0, help="NEXT f3 (1 closed loop) / f4 (2 gradual)")
     ap.add_argument("--step", type=int, default=1, help="ratio step of the gradual variant")
     ap.add_argument("--burst", type=float, default=0.0,
@@ -409,6 +475,8 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    if args.bound > 0 and args.impl == "ours":
+        return run_bound(args)
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)

@@ -281,8 +281,10 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
   const int64_t per_seg = (int64_t)ngroups * nbund;
   const int64_t s = ticket / per_seg;
   const int32_t rem = (int32_t)(ticket - s * per_seg);
-  const int32_t bidx = rem / ngroups;
-  const int32_t g = rem % ngroups;
+  // bundles of one (segment, group) take consecutive tickets, so they start
+  // together and stream the same trace tiles while those are still in L2
+  const int32_t bidx = rem % nbund;
+  const int32_t g = rem / nbund;
   int32_t cfg[NB];
 #pragma unroll
   for (int k = 0; k < NB; ++k) cfg[k] = bundles[bidx * NB + k];  // global config, -1 = pad
