@@ -49,6 +49,8 @@ struct magus_ctx_s {
   int64_t opt_bundle = 0;           // 0 auto, else force NB in {1, 2, 4}
   int64_t uploaded_bundle_opt = -1;
   // e2e staging (device)
+  void* mul_dev = nullptr;  // digest multiplier table mix64(w) | 1, w < mul_nw
+  int64_t mul_nw = 0;
   void* lam_dev = nullptr;  // NEXT f2 lambda grid
   size_t lam_bytes = 0;
   void* stage_dev = nullptr;
@@ -230,6 +232,19 @@ magus_status encode_tmap(magus_ctx ctx, CUtensorMap* map, const float* x, int64_
                            estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
                            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return fail(ctx, MAGUS_ERR_CUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  return MAGUS_OK;
+}
+
+// 1-D map over the digest table: one 16-B box (2 x u64) per decision word
+magus_status encode_mul_tmap(magus_ctx ctx, CUtensorMap* map) {
+  cuuint64_t dims[1] = {(cuuint64_t)(2 * ctx->mul_nw)};
+  cuuint64_t strides[1] = {(cuuint64_t)(2 * ctx->mul_nw) * 8};  // rank 1: not read
+  cuuint32_t box[1] = {2};
+  cuuint32_t estr[1] = {1};
+  CUresult r = ctx->encode(map, CU_TENSOR_MAP_DATA_TYPE_UINT64, 1, ctx->mul_dev, dims, strides, box, estr,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                           CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(ctx, MAGUS_ERR_CUDA, "digest tensor map failed (%d)", (int)r);
   return MAGUS_OK;
 }
 
@@ -442,6 +457,7 @@ magus_status magus_destroy(magus_ctx ctx) {
     if (ctx->pol_host) cudaFreeHost(ctx->pol_host);
     if (ctx->best_pinned) cudaFreeHost(ctx->best_pinned);
     if (ctx->lam_dev) cudaFree(ctx->lam_dev);
+    if (ctx->mul_dev) cudaFree(ctx->mul_dev);
     if (ctx->stage_dev) cudaFree(ctx->stage_dev);
     if (ctx->pol_copied) cudaEventDestroy(ctx->pol_copied);
     for (auto& pr : ctx->pending) {
@@ -610,15 +626,30 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     wk.dec = out_decisions;
     wk.dec_cstride = nw * N;
     wk.totals = out_totals;
-    CUtensorMap map;
+    if (nw > ctx->mul_nw) {  // the table depends on w only: grow it once, keep it
+      CK(cudaStreamSynchronize(ctx->stream));
+      if (ctx->mul_dev) cudaFree(ctx->mul_dev);
+      ctx->mul_dev = nullptr;
+      ctx->mul_nw = 0;
+      const int64_t cap = std::max<int64_t>(nw, 4096);
+      CK(cudaMalloc(&ctx->mul_dev, 2 * sizeof(unsigned long long) * (size_t)cap));
+      if (launch_digest_table(ctx->stream, (unsigned long long*)ctx->mul_dev, cap) < 0)
+        return cuda_fail(ctx, cudaGetLastError(), "digest table launch");
+      ctx->launches += 1;
+      ctx->mul_nw = cap;
+    }
+    wk.mul = (const unsigned long long*)ctx->mul_dev;
+    CUtensorMap map, map_mul;
     st = encode_tmap(ctx, &map, traces, N, T, ld);
+    if (st != MAGUS_OK) return st;
+    st = encode_mul_tmap(ctx, &map_mul);
     if (st != MAGUS_OK) return st;
     if (ctx->opt_timing) CK(cudaEventRecord(ev0, ctx->stream));
     int64_t grid_total = 0;
     for (size_t gi = 0; gi < ctx->groups.size(); ++gi) {
       auto& g = ctx->groups[gi];
       int grid = 0;
-      int r = launch_stream(ctx->stream, &map, N, T, dev_policies(ctx), dev_cidx(ctx, g.off), g.nbund,
+      int r = launch_stream(ctx->stream, &map, &map_mul, N, T, dev_policies(ctx), dev_cidx(ctx, g.off), g.nbund,
                             g.NB, g.W, g.H, ctx->dplat, nseg, seg_len, wk, &grid);
       if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "stream kernel launch");
       launched += r;

@@ -79,6 +79,19 @@ gen_kernel(uint64_t seed, int64_t id0, int64_t N, int64_t T, int64_t ld, int32_t
   for (int64_t t = 0; t < T; ++t) out[t * ld + i] = (float)mg_step(&g);
 }
 
+__global__ void digest_table_kernel(unsigned long long* __restrict__ mul, int64_t nw) {
+  const int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (w < nw) {  // 16-B rows so the stream kernel can bulk-copy one per stage
+    mul[2 * w] = digest_mul(w);
+    mul[2 * w + 1] = 0ULL;
+  }
+}
+
+int launch_digest_table(cudaStream_t s, unsigned long long* mul, int64_t nw) {
+  digest_table_kernel<<<(unsigned)((nw + 255) / 256), 256, 0, s>>>(mul, nw);
+  return cudaGetLastError() == cudaSuccess ? 1 : -1;
+}
+
 int launch_gen(cudaStream_t s, uint64_t seed, int64_t id0, int64_t N, int64_t T, int64_t ld,
                int32_t kind, float* out) {
   gen_kernel<<<(unsigned)((N + 127) / 128), 128, 0, s>>>(seed, id0, N, T, ld, kind, out);

@@ -81,6 +81,14 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, u
       "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
       : "memory");
 }
+__device__ __forceinline__ void tma_load_1d(void* dst, const CUtensorMap* map, uint64_t* bar,
+                                            int32_t c0) {
+  asm volatile(
+      "cp.async.bulk.tensor.1d.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3}], [%2];" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0)
+      : "memory");
+}
 __device__ __forceinline__ void st_release(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
@@ -245,7 +253,8 @@ struct BundleSmem {  // rarely touched, per (config slot, thread)
 
 template <int W_T, int H_T, int NB, bool BURST>
 __global__ void __launch_bounds__(kThreads, Occ<W_T, NB>::v)
-stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
+stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ CUtensorMap tmul,
+              int64_t N, int64_t T,
               const DevPolicy* __restrict__ pol, const int32_t* __restrict__ bundles, DevPlatform plat,
               int64_t nseg, int64_t seg_len, int32_t ngroups, int32_t nbund, StreamWork wk) {
   constexpr int kStages = Stages<W_T>::n;
@@ -254,11 +263,12 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
   __shared__ __align__(8) uint64_t full_bar[kStages];
   __shared__ __align__(8) uint64_t empty_bar[kStages];
   __shared__ uint32_t sh_ticket, sh_last, sh_last2;
-  // per-stage word constants, computed by the producer lane off the critical path
-  __shared__ unsigned long long st_mul[kStages];  // digest multiplier mix64(w) | 1
-  __shared__ uint32_t st_warm[kStages];           // positions t < W (no MDFS round yet)
-  __shared__ uint32_t st_tail[kStages];           // positions t < T
   __shared__ unsigned long long sh_red[kConsumerWarps][kTotAcc];
+  // digest multiplier of each staged word, delivered by a 16-B bulk copy from
+  // the context's table on the stage's own full barrier (async proxy, like
+  // the samples; generic-proxy stores here would race the consumers' reads)
+  // (tensor-copy destinations are 128-B aligned: one 128-B slot per stage)
+  __shared__ __align__(128) unsigned long long st_mul[kStages][16];
   __shared__ BundleSmem bs[NB][kTraces];
 
   if (threadIdx.x == 0) {
@@ -311,11 +321,8 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
       uint32_t ph = 0;
       for (int32_t j = 0; j < nwords; ++j) {
         if (j >= kStages) mbar_wait(&empty_bar[st], ph ^ 1u);
-        const int32_t w = w_first + j, p0 = w * 32;
-        st_mul[st] = digest_mul(w);
-        st_warm[st] = (p0 >= W) ? 0u : ((W - p0) >= 32 ? ~0u : ((1u << (W - p0)) - 1u));
-        st_tail[st] = tail_mask(p0, T);
-        mbar_expect_tx(&full_bar[st], kStageBytes);  // arrive: releases the writes above
+        mbar_expect_tx(&full_bar[st], kStageBytes + 16u);
+        tma_load_1d(st_mul[st], &tmul, &full_bar[st], 2 * (w_first + j));
         tma_load_2d(sm + st * kStageFloats, &tmap, &full_bar[st], g * kTraces,
                     (int32_t)((w_first + j) * kRows));
         if (++st == kStages) { st = 0; ph ^= 1u; }
@@ -398,14 +405,15 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
         wmax = fmaxf(wmax, xi);
       }
     }
-    const uint32_t warm = st_warm[st];
+    // warp-uniform word constants (kept in uniform registers by the compiler)
+    const uint32_t warm = (p0 >= W) ? 0u : ((W - p0) >= 32 ? ~0u : ((1u << (W - p0)) - 1u));
     const uint32_t incv = incw & ~warm;          // p = +1
     const uint32_t decv = decw & ~warm & ~incv;  // p = -1 (line 4 before line 6)
     const uint32_t E = incv | decv;              // uncore_tune_ls.push_back(1)
 
     if (w >= wt0) {
-      const uint32_t outm = st_tail[st];
-      const uint64_t M = st_mul[st];
+      const uint32_t outm = tail_mask(p0, T);
+      const uint64_t M = st_mul[st][0];       // digest multiplier mix64(w) | 1
       const bool final_word = (w == wend - 1);
       ev += __popc(E & outm);
       uint32_t bb = 0;  // bursts at max uncore: delivered x > theta
@@ -682,7 +690,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, int64_t N, int64_t T,
   }
 }
 
-typedef void (*stream_fn)(CUtensorMap, int64_t, int64_t, const DevPolicy*, const int32_t*,
+typedef void (*stream_fn)(CUtensorMap, CUtensorMap, int64_t, int64_t, const DevPolicy*, const int32_t*,
                           DevPlatform, int64_t, int64_t, int32_t, int32_t, StreamWork);
 
 struct Pick {
@@ -735,7 +743,7 @@ int stream_ctas_per_sm(int32_t W, int32_t H, int32_t NB) {
   return nb;
 }
 
-int launch_stream(cudaStream_t st, const void* tmap, int64_t N, int64_t T,
+int launch_stream(cudaStream_t st, const void* tmap, const void* tmap_mul, int64_t N, int64_t T,
                   const DevPolicy* pol_dev, const int32_t* bundles_dev, int32_t nbund, int32_t NB,
                   int32_t W, int32_t H, const DevPlatform& plat, int64_t nseg, int64_t seg_len,
                   const StreamWork& wk, int* grid_out) {
@@ -746,7 +754,8 @@ int launch_stream(cudaStream_t st, const void* tmap, int64_t N, int64_t T,
   const int64_t grid = (int64_t)ngroups * nseg * nbund;
   if (grid_out) *grid_out = (int)grid;
   const CUtensorMap* m = reinterpret_cast<const CUtensorMap*>(tmap);
-  p.f<<<(unsigned)grid, kThreads, p.smem, st>>>(*m, N, T, pol_dev, bundles_dev, plat, nseg, seg_len,
+  const CUtensorMap* mm = reinterpret_cast<const CUtensorMap*>(tmap_mul);
+  p.f<<<(unsigned)grid, kThreads, p.smem, st>>>(*m, *mm, N, T, pol_dev, bundles_dev, plat, nseg, seg_len,
                                                 ngroups, nbund, wk);
   return cudaGetLastError() == cudaSuccess ? 1 : -1;
 }

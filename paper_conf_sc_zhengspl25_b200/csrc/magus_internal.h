@@ -66,7 +66,8 @@ struct StreamWork {
   magus_base* base;              // [N] or NULL
   uint32_t* dec;                 // [C][nw][N] or NULL
   int64_t dec_cstride;           // nw * N
-  uint64_t* totals;              // [C][16] or NULL
+  uint64_t* totals;              // [C][18] or NULL
+  const unsigned long long* mul; // [ceil(T/32)][2] {mix64(w) | 1, 0}: 16-B bulk-copy rows
 };
 
 // Host precompute (precompute.cpp); returns false + message on invalid input.
@@ -94,7 +95,8 @@ bool stream_supported(int32_t W, int32_t H);
 // [nbund][NB] global config indices, -1 = padding).  All configs of a launch
 // share (W, H); the configs of a bundle also share L, tau_inc and tau_dec.
 // Replay + carry look-back + finalisation + totals in one launch.
-int launch_stream(cudaStream_t s, const void* tmap /* CUtensorMap, host copy */, int64_t N,
+int launch_stream(cudaStream_t s, const void* tmap /* CUtensorMap, host copy */,
+                  const void* tmap_mul /* CUtensorMap over StreamWork::mul */, int64_t N,
                   int64_t T, const DevPolicy* pol_dev, const int32_t* bundles_dev, int32_t nbund,
                   int32_t NB, int32_t W, int32_t H, const DevPlatform& plat, int64_t nseg,
                   int64_t seg_len, const StreamWork& wk, int* grid_out);
@@ -107,6 +109,9 @@ int launch_bound(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t l
 
 int launch_totals(cudaStream_t s, const magus_summary* summary, const magus_base* base, int64_t N,
                   int64_t T, int32_t C, uint64_t* totals);
+
+// digest multiplier table mul[w] = mix64(w) | 1 for w < nw (kernels_post.cu)
+int launch_digest_table(cudaStream_t s, unsigned long long* mul, int64_t nw);
 
 int launch_gen(cudaStream_t s, uint64_t seed, int64_t id0, int64_t N, int64_t T, int64_t ld,
                int32_t kind, float* out);

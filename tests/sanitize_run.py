@@ -1,0 +1,54 @@
+"""Small replay workload for compute-sanitizer (memcheck / racecheck /
+synccheck / initcheck) runs of the TMA + mbarrier + look-back kernels.
+
+  compute-sanitizer --tool racecheck python tests/sanitize_run.py
+
+Exercises: several segments (look-back), a ragged trace group and tail word,
+bundles (NB = 4), bursts, decisions output, the per-sample kernel and the DP.
+Exits non-zero if the results disagree with the oracle.
+"""
+import os
+import sys
+
+import numpy as np
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import gen  # noqa: E402
+import oracle  # noqa: E402
+import torch  # noqa: E402
+
+import paper_conf_sc_zhengspl25_b200 as magus  # noqa: E402
+
+
+def main():
+    N, T = 200, 1500
+    x = gen.gen_traces(gen.SEEDS[1], N, T)
+    xd = torch.zeros((T, 200), dtype=torch.float32, device="cuda:0")
+    xd[:, :N] = torch.from_numpy(x).cuda()
+    pols = [magus.make_policy(t_hi=th) for th in (0.2, 0.3, 0.4)] + [magus.make_policy(W=7, H=13)]
+    plat = magus.platform_preset()
+    plat.burst_mbs = 12000.0
+    po = oracle.policies([dict(W=p.window, H=p.history, L=p.deriv_len, tau_inc=p.tau_inc, tau_dec=p.tau_dec,
+                               t_hi=p.t_hi) for p in pols])
+    ref = oracle.replay(x, po, oracle.platform(burst=12000.0), want_dec=True)
+    ok = True
+    with magus.Context(device=0, platform=plat) as ctx:
+        for kernel, segs in ((magus.KERNEL_STREAM, 5), (magus.KERNEL_REFERENCE, 0)):
+            ctx.set_option(magus.OPT_KERNEL, kernel)
+            ctx.set_option(magus.OPT_SEGMENTS, segs)
+            r = ctx.replay(xd, pols, n_traces=N, want_decisions=True)
+            torch.cuda.synchronize()
+            got = r.summary_numpy()
+            ok &= bool(np.array_equal(got["energy_j"], ref.summary["energy"]))
+            ok &= bool(np.array_equal(got["digest"], ref.summary["digest"]))
+            ok &= bool(np.array_equal(r.decisions_numpy().transpose(0, 2, 1), oracle.decision_words(ref.dec, 8)))
+        out = ctx.offline_bound(xd[:200, :8], [0.0, 100.0])
+        torch.cuda.synchronize()
+        ok &= bool(np.array_equal(out.cpu().numpy()[3, 1], oracle.offline_bound(x[:200, 3], 100.0)))
+    print("sanitize workload parity:", "ok" if ok else "MISMATCH")
+    return 0 if ok else 1
+
+
+if __name__ == "__main__":
+    sys.exit(main())
