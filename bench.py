@@ -238,13 +238,24 @@ def run_ours(args):
     torch.cuda.synchronize()
 
     out = None
+    sweep_buf = None
 
     def step():
-        nonlocal out
+        # replay (one fused launch per W group) -> NCCL sum of the integer
+        # totals -> device-side choice + async device->host copy of the result
+        # into pinned memory (no host sync inside a step; --sync-sweep restores
+        # the synchronous magus_sweep_best)
+        nonlocal out, sweep_buf
         out = ctx.replay(x, pols, want_summary=False, want_base=False, want_decisions=want_dec,
                          want_totals=True, out=out)
         mdist.allreduce_totals(out.totals)  # the one collective; exact (integer words)
-        return ctx.sweep_best(out.totals)
+        if args.sync_sweep:
+            return ctx.sweep_best(out.totals)
+        sweep_buf = ctx.sweep_best_async(out.totals, sweep_buf)
+        return sweep_buf
+
+    def result(r):
+        return r if args.sync_sweep else ctx.sweep_result(r)
 
     for _ in range(args.warmup):
         step()
@@ -265,6 +276,7 @@ def run_ours(args):
         best = step()
     e1.record(stream)
     torch.cuda.synchronize()
+    best = result(best)
     clocks.mark()
     if world > 1:
         dist.barrier()
@@ -461,6 +473,8 @@ def main():
     ap.add_argument("--waves", type=int, default=0, help="MAGUS_OPT_WAVES (0 = library default)")
     ap.add_argument("--segments", type=int, default=0, help="MAGUS_OPT_SEGMENTS (0 = auto)")
     ap.add_argument("--bundle", type=int, default=0, help="MAGUS_OPT_BUNDLE (0 = auto, 1, 2, 4)")
+    ap.add_argument("--sync-sweep", action="store_true",
+                    help="host-synchronous magus_sweep_best each step (default: the async device choice)")
     ap.add_argument("--bound", type=int, default=0,
                     help="NEXT f2: time magus_offline_bound with this many lambdas instead of the replay")
     ap.add_argument("--full-grid", action="store_true", help="f2 over every ratio, not {min, max}")

@@ -280,6 +280,19 @@ magus_status magus_sweep_best(magus_ctx ctx, const uint64_t* totals,
                               int32_t n_params, int32_t* best,
                               magus_derived* best_row);
 
+/* Asynchronous form of magus_sweep_best: the derivation and the argmin run
+ * on the device (bit-identical to the host derivation) and the result is
+ * copied to host memory in ONE transfer without synchronising the stream;
+ * *out is valid once the stream reaches this point (pinned host memory
+ * keeps the copy asynchronous). */
+typedef struct {
+  int32_t best;           /* chosen config (argmin (n_viol, energy) if none feasible) */
+  int32_t feasible;       /* 1 if some config has n_viol == 0                        */
+  magus_derived row;      /* its fleet quantities                                    */
+} magus_choice;
+magus_status magus_sweep_best_async(magus_ctx ctx, const uint64_t* totals, int32_t n_params,
+                                    magus_choice* out);
+
 /* Host-only forms (no context, no GPU): the same derivation and choice from
  * host totals [n_params][MAGUS_TOT_WORDS] under *plat.  Used by the
  * multi-rank glue after the all-reduce and by CPU tests. */

@@ -58,6 +58,10 @@ class Derived(ctypes.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
+class Choice(ctypes.Structure):
+    _fields_ = [("best", ctypes.c_int32), ("feasible", ctypes.c_int32), ("row", Derived)]
+
+
 class PolicyConsts(ctypes.Structure):
     _fields_ = [("delta_inc", ctypes.c_double), ("delta_dec", ctypes.c_double), ("k_hi", ctypes.c_int32),
                 ("reserved", ctypes.c_int32)]
@@ -100,6 +104,7 @@ _lib.magus_replay.argtypes = [_vp, _vp, _i64, _i64, _i64, ctypes.POINTER(Policy)
 _lib.magus_replay_host.argtypes = [_vp, _vp, _i64, _i64, _i64, ctypes.POINTER(Policy), _i32, _vp, _vp, _vp, _vp]
 _lib.magus_replay_levels.argtypes = [_vp, _vp, _i64, _i64, _i64, ctypes.POINTER(Policy), _i32, _vp, _vp, _vp]
 _lib.magus_offline_bound.argtypes = [_vp, _vp, _i64, _i64, _i64, _vp, _i32, _i32, _vp]
+_lib.magus_sweep_best_async.argtypes = [_vp, _vp, _i32, _vp]
 _lib.magus_totals_derive.argtypes = [_vp, _vp, ctypes.POINTER(Derived)]
 _lib.magus_sweep_best.argtypes = [_vp, _vp, _i32, ctypes.POINTER(_i32), ctypes.POINTER(Derived)]
 _lib.magus_gen_traces.argtypes = [_vp, _u64, _i64, _i64, _i64, _i64, _i32, _vp]
@@ -118,7 +123,7 @@ for _f in ("magus_init", "magus_destroy", "magus_set_stream", "magus_policy_pres
            "magus_totals_derive", "magus_sweep_best", "magus_gen_traces", "magus_set_option",
            "magus_get_stats", "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
            "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host",
-           "magus_replay_levels", "magus_offline_bound"):
+           "magus_replay_levels", "magus_offline_bound", "magus_sweep_best_async"):
     getattr(_lib, _f).restype = ctypes.c_int
 
 EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_string", "magus_last_error",
@@ -127,7 +132,7 @@ EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_str
             "magus_sweep_best", "magus_gen_traces", "magus_set_option", "magus_get_stats",
             "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
             "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host",
-            "magus_replay_levels", "magus_offline_bound"]
+            "magus_replay_levels", "magus_offline_bound", "magus_sweep_best_async"]
 VARIANT_CLOSED_LOOP, VARIANT_GRADUAL = 1, 2
 
 
@@ -410,6 +415,21 @@ class Context:
         st = _lib.magus_pareto_front(self._h, _vp(totals.data_ptr()), C, _vp(on.ctypes.data), ctypes.byref(nf))
         self._check(st, "pareto_front")
         return on.astype(bool)
+
+    def sweep_best_async(self, totals, out=None):
+        """Enqueue the device-side choice (one D2H copy of a magus_choice into
+        a pinned buffer, returned); read it with sweep_result() after a sync."""
+        torch = self._torch
+        if out is None:
+            out = torch.zeros(ctypes.sizeof(Choice), dtype=torch.uint8, pin_memory=True)
+        st = _lib.magus_sweep_best_async(self._h, _vp(totals.data_ptr()), totals.shape[0], _vp(out.data_ptr()))
+        self._check(st, "sweep_best_async")
+        return out
+
+    @staticmethod
+    def sweep_result(out) -> tuple[int, dict, bool]:
+        ch = Choice.from_buffer_copy(out.numpy().tobytes())
+        return int(ch.best), ch.row.as_dict(), bool(ch.feasible)
 
     def sweep_best(self, totals) -> tuple[int, dict, bool]:
         """totals: CUDA int64 tensor [C, 16] (summed over ranks if sharded).

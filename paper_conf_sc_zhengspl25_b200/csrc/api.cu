@@ -49,6 +49,7 @@ struct magus_ctx_s {
   int64_t opt_bundle = 0;           // 0 auto, else force NB in {1, 2, 4}
   int64_t uploaded_bundle_opt = -1;
   // e2e staging (device)
+  void* sweep_dev = nullptr;  // SweepResult of magus_sweep_best_async
   void* mul_dev = nullptr;  // digest multiplier table mix64(w) | 1, w < mul_nw
   int64_t mul_nw = 0;
   void* lam_dev = nullptr;  // NEXT f2 lambda grid
@@ -458,6 +459,7 @@ magus_status magus_destroy(magus_ctx ctx) {
     if (ctx->best_pinned) cudaFreeHost(ctx->best_pinned);
     if (ctx->lam_dev) cudaFree(ctx->lam_dev);
     if (ctx->mul_dev) cudaFree(ctx->mul_dev);
+    if (ctx->sweep_dev) cudaFree(ctx->sweep_dev);
     if (ctx->stage_dev) cudaFree(ctx->stage_dev);
     if (ctx->pol_copied) cudaEventDestroy(ctx->pol_copied);
     for (auto& pr : ctx->pending) {
@@ -834,6 +836,20 @@ magus_status magus_pareto_front_host(const magus_platform* plat, const uint64_t*
   if (!plat || !totals_host || C < 1 || !on_front || !validate_platform(*plat, msg, sizeof msg))
     return MAGUS_ERR_INVALID_ARG;
   pareto(make_dev_platform(*plat), totals_host, C, on_front, n_front);
+  return MAGUS_OK;
+}
+
+magus_status magus_sweep_best_async(magus_ctx ctx, const uint64_t* totals, int32_t C,
+                                    magus_choice* out) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  if (!totals || C < 1 || !out) return fail(ctx, MAGUS_ERR_INVALID_ARG, "bad sweep_best_async arguments");
+  DeviceGuard dg(ctx->device);
+  if (!ctx->sweep_dev) CK(cudaMalloc(&ctx->sweep_dev, sizeof(SweepResult)));
+  SweepResult* r = (SweepResult*)ctx->sweep_dev;
+  if (launch_sweep_best(ctx->stream, totals, C, ctx->dplat, r) < 0)
+    return cuda_fail(ctx, cudaGetLastError(), "sweep_best kernel launch");
+  ctx->launches += 1;
+  CK(cudaMemcpyAsync(out, r, sizeof(magus_choice), cudaMemcpyDeviceToHost, ctx->stream));
   return MAGUS_OK;
 }
 

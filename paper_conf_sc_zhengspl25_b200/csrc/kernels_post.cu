@@ -79,6 +79,78 @@ gen_kernel(uint64_t seed, int64_t id0, int64_t N, int64_t T, int64_t ld, int32_t
   for (int64_t t = 0; t < T; ++t) out[t * ld + i] = (float)mg_step(&g);
 }
 
+// ---------------------------------------------------------------------------
+// Device form of the fleet derivation + sweep choice (api.cu derive_totals /
+// choose_best), bit-identical: the same fp64 operations in the same order,
+// and a correctly rounded conversion of the 128-bit q sums to double.
+// ---------------------------------------------------------------------------
+// RN(unsigned 128-bit hi:lo) to double: keep the top 64 bits, fold every
+// dropped bit into a sticky LSB (below the rounding position), convert, scale.
+__device__ __forceinline__ double u128_to_double_rn(uint64_t hi, uint64_t lo) {
+  if (hi == 0) return __ull2double_rn(lo);
+  const int s = 64 - __clzll(hi);                     // bits beyond the low 64, 1..64
+  const uint64_t top = s == 64 ? hi : ((hi << (64 - s)) | (lo >> s));  // the top 64 bits
+  const uint64_t sticky = (s == 64 ? lo : (lo << (64 - s))) != 0 ? 1ULL : 0ULL;
+  return ldexp(__ull2double_rn(top | sticky), s);
+}
+// Q = qhi_sum * 2^32 + qlo_sum as a 128-bit value
+__device__ __forceinline__ void limbs_to_u128(uint64_t hi_sum, uint64_t lo_sum, uint64_t& H, uint64_t& L) {
+  const uint64_t a = hi_sum << 32;
+  L = a + lo_sum;
+  H = (hi_sum >> 32) + (L < a ? 1ULL : 0ULL);
+}
+__device__ void derive_dev(const DevPlatform& p, const uint64_t* w, magus_derived* out) {
+  const uint64_t NT = w[MAGUS_TOT_N_STEPS], mint = w[MAGUS_TOT_MIN_INT];
+  uint64_t h1, l1, h2, l2, h3, l3;
+  limbs_to_u128(w[MAGUS_TOT_QMIN_HI], w[MAGUS_TOT_QMIN_LO], h1, l1);
+  limbs_to_u128(w[MAGUS_TOT_QMAX_HI], w[MAGUS_TOT_QMAX_LO], h2, l2);
+  limbs_to_u128(w[MAGUS_TOT_QBASE_HI], w[MAGUS_TOT_QBASE_LO], h3, l3);
+  const uint64_t ls = l1 + l2, hs = h1 + h2 + (ls < l1 ? 1ULL : 0ULL);  // qmin + qmax
+  const double ch = (double)w[MAGUS_TOT_CHANGES];
+  const double time_max = p.dt * (double)(NT - mint) + p.cQ * u128_to_double_rn(h2, l2);
+  const double time_min = p.dt * (double)mint + p.cQ * u128_to_double_rn(h1, l1);
+  const double time = (p.dt * (double)NT + p.cQ * u128_to_double_rn(hs, ls)) + p.t_sw * ch;
+  const double energy = (p.P_max * time_max + p.P_min * time_min) + p.e_sw * ch;
+  const double base_time = p.dt * (double)NT + p.cQ * u128_to_double_rn(h3, l3);
+  const double base_energy = p.P_max * base_time;
+  out->energy_j = energy;
+  out->time_s = time;
+  out->base_energy_j = base_energy;
+  out->base_time_s = base_time;
+  out->saving = 1.0 - energy / base_energy;
+  out->slowdown = time / base_time - 1.0;
+  out->n_viol = (int64_t)w[MAGUS_TOT_N_VIOL];
+  out->n_traces = (int64_t)w[MAGUS_TOT_N_TRACES];
+  const uint64_t uni = w[MAGUS_TOT_BURST_BASE], inter = w[MAGUS_TOT_BURST_MAGUS];
+  out->jaccard = uni ? (double)inter / (double)uni : 1.0;
+}
+
+// one thread: C <= a few hundred configs, a handful of fp64 ops each
+__global__ void sweep_best_kernel(const uint64_t* __restrict__ tot, int32_t C, DevPlatform plat,
+                                  SweepResult* __restrict__ res) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  int32_t b = -1, bi = 0;
+  magus_derived db, di, dc;
+  derive_dev(plat, tot, &di);  // infeasible fallback: argmin (n_viol, energy)
+  for (int32_t c = 0; c < C; ++c) {
+    derive_dev(plat, tot + (int64_t)c * MAGUS_TOT_WORDS, &dc);
+    if (dc.n_viol == 0 && (b < 0 || dc.energy_j < db.energy_j)) { b = c; db = dc; }
+    if (c > 0 && (dc.n_viol < di.n_viol || (dc.n_viol == di.n_viol && dc.energy_j < di.energy_j))) {
+      bi = c;
+      di = dc;
+    }
+  }
+  res->feasible = b >= 0 ? 1 : 0;
+  res->best = b >= 0 ? b : bi;
+  res->row = b >= 0 ? db : di;
+}
+
+int launch_sweep_best(cudaStream_t s, const uint64_t* totals, int32_t C, const DevPlatform& plat,
+                      SweepResult* res) {
+  sweep_best_kernel<<<1, 32, 0, s>>>(totals, C, plat, res);
+  return cudaGetLastError() == cudaSuccess ? 1 : -1;
+}
+
 __global__ void digest_table_kernel(unsigned long long* __restrict__ mul, int64_t nw) {
   const int64_t w = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (w < nw) {  // 16-B rows so the stream kernel can bulk-copy one per stage

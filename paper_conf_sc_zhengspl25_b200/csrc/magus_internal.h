@@ -110,6 +110,11 @@ int launch_bound(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t l
 int launch_totals(cudaStream_t s, const magus_summary* summary, const magus_base* base, int64_t N,
                   int64_t T, int32_t C, uint64_t* totals);
 
+// device sweep choice (kernels_post.cu), bit-identical to the host form
+typedef magus_choice SweepResult;
+int launch_sweep_best(cudaStream_t s, const uint64_t* totals, int32_t C, const DevPlatform& plat,
+                      SweepResult* res);
+
 // digest multiplier table mul[w] = mix64(w) | 1 for w < nw (kernels_post.cu)
 int launch_digest_table(cudaStream_t s, unsigned long long* mul, int64_t nw);
 
