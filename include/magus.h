@@ -230,6 +230,41 @@ magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t n_traces,
                           magus_summary* out_summary, magus_base* out_base,
                           uint32_t* out_decisions, uint64_t* out_totals);
 
+/* ---- time-chunked replay (SURVEY §8(b) magus_replay_resume, §8(e)) -----
+ * Replays a long trace set in time chunks that need not fit in HBM together
+ * (config 4: 262 GB on one GPU).  Exact by the closed form of Alg. 3
+ * (DESIGN.md 6.3): p_t and the Alg. 2 history depend only on
+ * x[t-W-H+1..t], and the only carried decision state is dec[t_start-1]; the
+ * model-M accumulators are integers, so chunk sums are order-free.
+ *
+ *   state     caller-owned DEVICE buffer of magus_resume_state_bytes(N, C)
+ *             bytes, 8-byte aligned, ALL ZERO before the first chunk (t = 0);
+ *             one state per (trace set, params) sequence; not shared between
+ *             concurrent calls.  Layout (opaque): integer accumulators
+ *             [C][12][N] u64, then dec[t_start-1] [C][N] u32.
+ *   traces    device, time-major like magus_replay: row r (< n_rows) holds
+ *             global interval t_base + r.
+ *   t_base    multiple of 32;  t_start multiple of 32 in [t_base,
+ *             t_base + n_rows): the first interval this call decides; it MUST
+ *             equal the end (t_base + n_rows) of the previous call on `state`
+ *             (0 on a zeroed state).  Rows [t_base, t_start) are the halo:
+ *             t_start - t_base >= min(t_start, magus_resume_halo(params)).
+ *             Chunks other than the last must end on a multiple of 32.
+ *   outputs   as magus_replay over the PREFIX [0, t_base + n_rows): summaries,
+ *             base and totals are those of a one-shot replay of the first
+ *             t_base + n_rows intervals (bit-identical); out_decisions holds
+ *             the words of [t_start, t_base + n_rows) only:
+ *             [n_params][ceil((t_base + n_rows - t_start)/32)][n_traces].
+ * Runs the stream kernel only (variant 0, W <= 33, H <= 32, 16-B aligned
+ * traces, ld % 4 == 0): MAGUS_ERR_UNSUPPORTED otherwise.  Asynchronous. */
+magus_status magus_resume_state_bytes(int64_t n_traces, int32_t n_params, size_t* out);
+magus_status magus_resume_halo(const magus_policy* params, int32_t n_params, int64_t* rows);
+magus_status magus_replay_resume(magus_ctx ctx, const float* traces, int64_t n_traces,
+                                 int64_t n_rows, int64_t ld, int64_t t_base, int64_t t_start,
+                                 const magus_policy* params, int32_t n_params, void* state,
+                                 magus_summary* out_summary, magus_base* out_base,
+                                 uint32_t* out_decisions, uint64_t* out_totals);
+
 /* Per-interval decisions as uncore ratios (needed for multi-level variants):
  * out_levels DEVICE uint8 [n_params][n_steps][n_traces], level[c][t][n] =
  * dec[t] of trace n under config c.  Runs the per-sample kernel; other

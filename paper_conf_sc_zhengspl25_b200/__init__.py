@@ -102,6 +102,10 @@ _lib.magus_grid_sweep256.argtypes = [ctypes.POINTER(Policy)]
 _lib.magus_grid_fleet64.argtypes = [ctypes.POINTER(Policy)]
 _lib.magus_replay.argtypes = [_vp, _vp, _i64, _i64, _i64, ctypes.POINTER(Policy), _i32, _vp, _vp, _vp, _vp]
 _lib.magus_replay_host.argtypes = [_vp, _vp, _i64, _i64, _i64, ctypes.POINTER(Policy), _i32, _vp, _vp, _vp, _vp]
+_lib.magus_replay_resume.argtypes = [_vp, _vp, _i64, _i64, _i64, _i64, _i64, ctypes.POINTER(Policy), _i32, _vp,
+                                     _vp, _vp, _vp, _vp]
+_lib.magus_resume_state_bytes.argtypes = [_i64, _i32, ctypes.POINTER(ctypes.c_size_t)]
+_lib.magus_resume_halo.argtypes = [ctypes.POINTER(Policy), _i32, ctypes.POINTER(_i64)]
 _lib.magus_replay_levels.argtypes = [_vp, _vp, _i64, _i64, _i64, ctypes.POINTER(Policy), _i32, _vp, _vp, _vp]
 _lib.magus_offline_bound.argtypes = [_vp, _vp, _i64, _i64, _i64, _vp, _i32, _i32, _vp]
 _lib.magus_sweep_best_async.argtypes = [_vp, _vp, _i32, _vp]
@@ -132,7 +136,8 @@ EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_str
             "magus_sweep_best", "magus_gen_traces", "magus_set_option", "magus_get_stats",
             "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
             "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host",
-            "magus_replay_levels", "magus_offline_bound", "magus_sweep_best_async"]
+            "magus_replay_levels", "magus_offline_bound", "magus_sweep_best_async",
+            "magus_replay_resume", "magus_resume_state_bytes", "magus_resume_halo"]
 VARIANT_CLOSED_LOOP, VARIANT_GRADUAL = 1, 2
 
 
@@ -173,6 +178,16 @@ def grid_fleet64() -> list[Policy]:
     arr = (Policy * 64)()
     _lib.magus_grid_fleet64(arr)
     return list(arr)
+
+
+def resume_halo(policies) -> int:
+    """Rows before t_start a resume chunk must carry (multiple of 32)."""
+    arr, C = _policy_array(policies)
+    r = _i64()
+    st = _lib.magus_resume_halo(arr, C, ctypes.byref(r))
+    if st:
+        raise MagusError(st, "resume_halo")
+    return r.value
 
 
 def policy_inspect(p: Policy) -> dict:
@@ -348,6 +363,40 @@ class Context:
         st = _lib.magus_replay(self._h, _vp(traces.data_ptr()), N, T, ld, arr, C, p(out.summary), p(out.base),
                                p(out.decisions), p(out.totals))
         self._check(st, "replay")
+        return out
+
+    def resume_state(self, n_traces: int, policies):
+        """Zeroed device resume state (t = 0) for replay_resume."""
+        _, C = _policy_array(policies)
+        nb = ctypes.c_size_t()
+        st = _lib.magus_resume_state_bytes(n_traces, C, ctypes.byref(nb))
+        self._check(st, "resume_state_bytes")
+        return self._torch.zeros(((nb.value + 7) // 8,), dtype=self._torch.int64, device=f"cuda:{self.device}")
+
+    def replay_resume(self, traces, policies, state, t_base: int, t_start: int, n_traces: int | None = None,
+                      want_summary: bool = True, want_base: bool = True, want_decisions: bool = False,
+                      want_totals: bool = True) -> ReplayResult:
+        """One time chunk: traces[r] = global interval t_base + r; decides
+        [t_start, t_base + rows); outputs cover the prefix [0, t_base + rows)."""
+        torch = self._torch
+        assert traces.is_cuda and traces.dtype == torch.float32 and traces.dim() == 2
+        assert traces.stride(1) == 1
+        R, ld = traces.shape[0], traces.stride(0)
+        N = traces.shape[1] if n_traces is None else n_traces
+        arr, C = _policy_array(policies)
+        dev = traces.device
+        nw = (t_base + R - t_start + 31) // 32
+        out = ReplayResult(
+            summary=torch.empty((C, N, SUMMARY_DT.itemsize), dtype=torch.uint8, device=dev) if want_summary else None,
+            base=torch.empty((N, 32), dtype=torch.uint8, device=dev) if want_base else None,
+            decisions=torch.empty((C, max(nw, 0), N), dtype=torch.int32, device=dev) if want_decisions else None,
+            totals=torch.empty((C, TOT_WORDS), dtype=torch.int64, device=dev) if want_totals else None,
+            n_traces=N, n_configs=C)
+        p = lambda t: _vp(t.data_ptr()) if t is not None else None  # noqa: E731
+        st = _lib.magus_replay_resume(self._h, _vp(traces.data_ptr()), N, R, ld, t_base, t_start, arr, C,
+                                      _vp(state.data_ptr()), p(out.summary), p(out.base), p(out.decisions),
+                                      p(out.totals))
+        self._check(st, "replay_resume")
         return out
 
     def replay_levels(self, traces, policies, n_traces: int | None = None, want_totals: bool = True):

@@ -505,13 +505,24 @@ magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value) {
   return fail(ctx, MAGUS_ERR_INVALID_ARG, "unknown option %d", key);
 }
 
+// time-chunked replay (magus_replay_resume): buffer row r = global interval
+// tb + r, output from row ts on, state = caller's resume state
+struct ResumeArgs {
+  int64_t tb, ts;
+  void* state;
+};
+
 static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, int64_t T,
                                 int64_t ld, const magus_policy* params, int32_t C,
                                 magus_summary* out_summary, magus_base* out_base,
-                                uint32_t* out_decisions, uint64_t* out_totals, uint8_t* out_levels) {
+                                uint32_t* out_decisions, uint64_t* out_totals, uint8_t* out_levels,
+                                const ResumeArgs* rs = nullptr) {
   if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
   magus_status st = validate_replay(ctx, traces, N, T, ld, params, C);
   if (st != MAGUS_OK) return st;
+  const int64_t tb = rs ? rs->tb : 0, ts = rs ? rs->ts : 0;
+  if (tb + T > kMaxSteps)
+    return fail(ctx, MAGUS_ERR_INVALID_ARG, "t_base + n_rows %lld exceeds 2^24", (long long)(tb + T));
   DeviceGuard dg(ctx->device);
   cudaGetLastError();
 
@@ -530,12 +541,17 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
   if (kernel == 2 && !(all_stream && tma_ok))
     return fail(ctx, MAGUS_ERR_UNSUPPORTED,
                 "stream kernel needs W in [2,33], H in [1,32], 16-B aligned traces and ld %% 4 == 0");
+  if (rs && kernel != 2)
+    return fail(ctx, MAGUS_ERR_UNSUPPORTED,
+                "time-chunked replay runs on the stream kernel only (variant 0, W in [2,33], "
+                "H in [1,32], 16-B aligned traces, ld %% 4 == 0)");
 
   st = upload_policies(ctx, params, C);
   if (st != MAGUS_OK) return st;
 
-  const int64_t nw = (T + 31) / 32;
-  int64_t nseg = 1, seg_len = ((T + 31) / 32) * 32;
+  const int64_t Tr = T - ts;            // rows this call replays
+  const int64_t nw = (Tr + 31) / 32;     // decision words written
+  int64_t nseg = 1, seg_len = ((Tr + 31) / 32) * 32;
   if (kernel == 2) {
     const int64_t ngroups = (N + 127) / 128;
     if (ctx->opt_segments > 0) {
@@ -551,13 +567,13 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
       const int64_t slots = (int64_t)ctx->sms * per_sm * ctx->opt_waves;
       nseg = std::max<int64_t>(1, (slots + ngroups * nbund - 1) / (ngroups * nbund));
     }
-    seg_len = ((T + nseg - 1) / nseg + 31) / 32 * 32;
+    seg_len = ((Tr + nseg - 1) / nseg + 31) / 32 * 32;
     bool packed = false;  // NB > 1 packs per-segment counters in 16 bits
     for (auto& g : ctx->groups) packed = packed || g.NB > 1;
     if (packed && seg_len > 65504) seg_len = 65504;
     const int64_t min_len = 512;  // keeps the halo re-read below ~6 %
-    if (ctx->opt_segments == 0 && seg_len < min_len) seg_len = std::min<int64_t>(min_len, ((T + 31) / 32) * 32);
-    nseg = (T + seg_len - 1) / seg_len;
+    if (ctx->opt_segments == 0 && seg_len < min_len) seg_len = std::min<int64_t>(min_len, ((Tr + 31) / 32) * 32);
+    nseg = (Tr + seg_len - 1) / seg_len;
   }
   const int64_t ngroups = (N + 127) / 128;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
@@ -628,12 +644,20 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     wk.dec = out_decisions;
     wk.dec_cstride = nw * N;
     wk.totals = out_totals;
-    if (nw > ctx->mul_nw) {  // the table depends on w only: grow it once, keep it
+    wk.tb = (int32_t)tb;       // global interval of buffer row 0
+    wk.ts = (int32_t)(tb + ts);  // first interval decided (global)
+    wk.carry = nullptr;
+    if (rs) {  // accumulators and carries live in the caller's state
+      wk.acc = (unsigned long long*)rs->state;
+      wk.carry = (uint32_t*)((char*)rs->state + 8 * (size_t)kAccFields * (size_t)(C * N));
+    }
+    const int64_t nw_glob = (tb + T + 31) / 32;  // digest words are global
+    if (nw_glob > ctx->mul_nw) {  // the table depends on w only: grow it once, keep it
       CK(cudaStreamSynchronize(ctx->stream));
       if (ctx->mul_dev) cudaFree(ctx->mul_dev);
       ctx->mul_dev = nullptr;
       ctx->mul_nw = 0;
-      const int64_t cap = std::max<int64_t>(nw, 4096);
+      const int64_t cap = std::max<int64_t>(nw_glob, 4096);
       CK(cudaMalloc(&ctx->mul_dev, 2 * sizeof(unsigned long long) * (size_t)cap));
       if (launch_digest_table(ctx->stream, (unsigned long long*)ctx->mul_dev, cap) < 0)
         return cuda_fail(ctx, cudaGetLastError(), "digest table launch");
@@ -651,7 +675,7 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     for (size_t gi = 0; gi < ctx->groups.size(); ++gi) {
       auto& g = ctx->groups[gi];
       int grid = 0;
-      int r = launch_stream(ctx->stream, &map, &map_mul, N, T, dev_policies(ctx), dev_cidx(ctx, g.off), g.nbund,
+      int r = launch_stream(ctx->stream, &map, &map_mul, N, tb + T, dev_policies(ctx), dev_cidx(ctx, g.off), g.nbund,
                             g.NB, g.W, g.H, ctx->dplat, nseg, seg_len, wk, &grid);
       if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "stream kernel launch");
       launched += r;
@@ -672,6 +696,53 @@ magus_status magus_replay(magus_ctx ctx, const float* traces, int64_t N, int64_t
                           magus_base* out_base, uint32_t* out_decisions, uint64_t* out_totals) {
   return replay_impl(ctx, traces, N, T, ld, params, C, out_summary, out_base, out_decisions,
                      out_totals, nullptr);
+}
+
+static int64_t resume_halo_rows(const magus_policy* params, int32_t C) {
+  int64_t h = 0;
+  for (int32_t c = 0; c < C; ++c)
+    h = std::max<int64_t>(h, ((int64_t)params[c].window + params[c].history - 1 + 31) / 32 * 32);
+  return h;
+}
+
+magus_status magus_resume_state_bytes(int64_t n_traces, int32_t n_params, size_t* out) {
+  if (!out || n_traces < 1 || n_params < 1) return MAGUS_ERR_INVALID_ARG;
+  *out = resume_state_bytes(n_traces, n_params);
+  return MAGUS_OK;
+}
+
+magus_status magus_resume_halo(const magus_policy* params, int32_t n_params, int64_t* rows) {
+  if (!params || n_params < 1 || !rows) return MAGUS_ERR_INVALID_ARG;
+  char msg[256];
+  for (int32_t c = 0; c < n_params; ++c)
+    if (!validate_policy(params[c], msg, sizeof msg)) return MAGUS_ERR_INVALID_ARG;
+  *rows = resume_halo_rows(params, n_params);
+  return MAGUS_OK;
+}
+
+magus_status magus_replay_resume(magus_ctx ctx, const float* traces, int64_t N, int64_t n_rows,
+                                 int64_t ld, int64_t t_base, int64_t t_start,
+                                 const magus_policy* params, int32_t C, void* state,
+                                 magus_summary* out_summary, magus_base* out_base,
+                                 uint32_t* out_decisions, uint64_t* out_totals) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  if (!state || (uintptr_t)state % 8 != 0)
+    return fail(ctx, MAGUS_ERR_INVALID_ARG, "state must be a non-NULL, 8-byte aligned device buffer");
+  if (t_base < 0 || t_base % 32 != 0 || t_start % 32 != 0)
+    return fail(ctx, MAGUS_ERR_INVALID_ARG, "t_base and t_start must be non-negative multiples of 32");
+  if (t_start < t_base || t_start >= t_base + n_rows)
+    return fail(ctx, MAGUS_ERR_INVALID_ARG, "t_start %lld outside the buffer [%lld, %lld)",
+                (long long)t_start, (long long)t_base, (long long)(t_base + n_rows));
+  if (params && C >= 1) {
+    const int64_t halo = std::min<int64_t>(t_start, resume_halo_rows(params, C));
+    if (t_start - t_base < halo)
+      return fail(ctx, MAGUS_ERR_INVALID_ARG,
+                  "the buffer must hold the %lld rows before t_start (t_base <= %lld)",
+                  (long long)halo, (long long)(t_start - halo));
+  }
+  const ResumeArgs rs{t_base, t_start - t_base, state};
+  return replay_impl(ctx, traces, N, n_rows, ld, params, C, out_summary, out_base, out_decisions,
+                     out_totals, nullptr, &rs);
 }
 
 magus_status magus_replay_levels(magus_ctx ctx, const float* traces, int64_t N, int64_t T,

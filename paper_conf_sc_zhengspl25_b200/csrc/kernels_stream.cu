@@ -243,7 +243,7 @@ struct BundleRegs {
   uint32_t cnt_f[NB];  // bursts kept under MAGUS (NB > 1: | prefix bursts << 16)
   uint32_t cnt_g[NB];  // NB == 1: bursts in the carry-dependent prefix
   unsigned long long qmin[NB], dig[NB], pqmin[NB];
-  uint32_t carry, seen, va, last;  // bit k per config
+  uint32_t carry, seen, va;  // bit k per config
 };
 struct BundleSmem {  // rarely touched, per (config slot, thread)
   unsigned long long qmax, pqmax, pdig;
@@ -262,7 +262,8 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   extern __shared__ __align__(1024) float sm[];
   __shared__ __align__(8) uint64_t full_bar[kStages];
   __shared__ __align__(8) uint64_t empty_bar[kStages];
-  __shared__ uint32_t sh_ticket, sh_last, sh_last2;
+  __shared__ uint32_t sh_last, sh_last2;
+  __shared__ int32_t sh_work[3];  // segment, bundle, group of this CTA
   __shared__ unsigned long long sh_red[kConsumerWarps][kTotAcc];
   // digest multiplier of each staged word, delivered by a 16-B bulk copy from
   // the context's table on the stage's own full barrier (async proxy, like
@@ -272,7 +273,17 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   __shared__ BundleSmem bs[NB][kTraces];
 
   if (threadIdx.x == 0) {
-    sh_ticket = atomicAdd(wk.ticket, 1u);  // launch-order work ticket
+    // launch-order work ticket -> (segment, bundle, group), segment-major so
+    // that the predecessor segment of the same (bundle, group) always holds a
+    // smaller ticket; bundles of one (segment, group) take consecutive
+    // tickets, so they start together and stream the same trace tiles while
+    // those are still in L2
+    const uint32_t ticket = atomicAdd(wk.ticket, 1u);
+    const uint32_t per_seg = (uint32_t)ngroups * (uint32_t)nbund;
+    const uint32_t sg = ticket / per_seg, rem = ticket - sg * per_seg;
+    sh_work[0] = (int32_t)sg;
+    sh_work[1] = (int32_t)(rem % (uint32_t)nbund);
+    sh_work[2] = (int32_t)(rem / (uint32_t)nbund);
     for (int i = 0; i < kStages; ++i) {
       mbar_init(&full_bar[i], 1);
       mbar_init(&empty_bar[i], kConsumerWarps);
@@ -285,32 +296,25 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   }
   __syncthreads();
 
-  // ticket -> (segment, bundle, group), segment-major so that the predecessor
-  // segment of the same (bundle, group) always holds a smaller ticket
-  const uint32_t ticket = sh_ticket;
-  const int64_t per_seg = (int64_t)ngroups * nbund;
-  const int64_t s = ticket / per_seg;
-  const int32_t rem = (int32_t)(ticket - s * per_seg);
-  // bundles of one (segment, group) take consecutive tickets, so they start
-  // together and stream the same trace tiles while those are still in L2
-  const int32_t bidx = rem % nbund;
-  const int32_t g = rem / nbund;
+  const int32_t s = sh_work[0];
+  const int32_t bidx = sh_work[1];
+  const int32_t g = sh_work[2];
   int32_t cfg[NB];
 #pragma unroll
   for (int k = 0; k < NB; ++k) cfg[k] = bundles[bidx * NB + k];  // global config, -1 = pad
   const int32_t c0 = cfg[0];
-  const int32_t t0 = (int32_t)(s * seg_len);  // T <= 2^24: time fits in 32 bits
+  // global intervals (T = end of this call, buffer row r = interval wk.tb + r);
+  // T <= 2^24: time fits in 32 bits
+  const int32_t t0 = wk.ts + (int32_t)(s * seg_len);
   const int32_t t1 = (int32_t)((t0 + seg_len < T) ? t0 + seg_len : T);
   const DevPolicy P = pol[c0];
   const int W = W_T > 0 ? W_T : P.W;
   const int H = H_T > 0 ? H_T : P.H;
   const int32_t wt0 = t0 >> 5;
   const int32_t wend = (t1 + 31) >> 5;
-  int32_t nhalo = 0;
-  if (s > 0) {
-    nhalo = (W + H - 1 + 31) / 32;
-    if (nhalo > wt0) nhalo = wt0;
-  }
+  const int32_t ws = wk.ts >> 5;  // first output word
+  int32_t nhalo = (W + H - 1 + 31) / 32;  // rows t0-W-H+1 .. t0-1 fix p and the history
+  if (nhalo > wt0 - (wk.tb >> 5)) nhalo = wt0 - (wk.tb >> 5);  // (none before the buffer)
   const int32_t w_first = wt0 - nhalo;
   const int32_t nwords = wend - w_first;
 
@@ -324,7 +328,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
         mbar_expect_tx(&full_bar[st], kStageBytes + 16u);
         tma_load_1d(st_mul[st], &tmul, &full_bar[st], 2 * (w_first + j));
         tma_load_2d(sm + st * kStageFloats, &tmap, &full_bar[st], g * kTraces,
-                    (int32_t)((w_first + j) * kRows));
+                    (int32_t)((w_first + j) * kRows - wk.tb));
         if (++st == kStages) { st = 0; ph ^= 1u; }
       }
     }
@@ -341,8 +345,15 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   for (int k = 0; k < NB; ++k) kk[k] = cfg[k] >= 0 ? pol[cfg[k]].k : 0x3F;
   const float xthr_min = plat.xthr_min, xthr_max = plat.xthr_max;
   const double invB24_min = plat.invB24_min, invB24_max = plat.invB24_max;
-  const uint32_t hyp = (s > 0) ? 1u : 0u;  // segment 0 starts from the true dec[-1] = max
-  const uint32_t last_bit = (uint32_t)((t1 - 1) & 31);
+  // carry hypothesis, bit k per config: later segments assume min; segment 0
+  // starts from the true dec[t_start-1] (max at t = 0, else the resume state)
+  // (re-read in the epilogue rather than kept live across the scan)
+  uint32_t hypm = (s > 0) ? (1u << NB) - 1u : 0u;
+  if (s == 0 && wk.carry && valid) {
+#pragma unroll
+    for (int k = 0; k < NB; ++k)
+      if (cfg[k] >= 0) hypm |= (__ldg(wk.carry + (int64_t)cfg[k] * N + n) & 1u) << k;
+  }
   BundleRegs<NB> B;
 #pragma unroll
   for (int k = 0; k < NB; ++k) {
@@ -352,15 +363,15 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
     bs[k][tid].qmax = 0; bs[k][tid].pqmax = 0; bs[k][tid].pdig = 0;
     bs[k][tid].apos = -1; bs[k][tid].wa = -1; bs[k][tid].dwa = 0; bs[k][tid].pre_dec_a = 0;
   }
-  B.carry = hyp ? (1u << NB) - 1u : 0u;
-  B.seen = 0; B.va = 0; B.last = 0;
+  B.carry = hypm;
+  B.seen = 0; B.va = 0;
   uint32_t Eprev = 0, ev = 0, bbase = 0;
   unsigned long long qbase = 0;
   constexpr bool bursts = BURST;                    // Sec. 6.3 Jaccard counters (f1)
   const bool bkeep = plat.burst_min_keeps != 0;     // B_min > theta: no burst is hidden
   const float xburst = plat.xburst;
   const bool want_dec = wk.dec != nullptr && valid;
-  uint32_t* dec_row = want_dec ? wk.dec + wt0 * N + n : nullptr;  // + c * dec_cstride
+  uint32_t* dec_row = want_dec ? wk.dec + (wt0 - ws) * N + n : nullptr;  // + c * dec_cstride
   double pd[W_T > 1 ? W_T - 1 : 1];  // previous word's last W-1 samples, widened
 #pragma unroll
   for (int k = 0; k < (W_T > 1 ? W_T - 1 : 1); ++k) pd[k] = 0.0;
@@ -414,7 +425,6 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
     if (w >= wt0) {
       const uint32_t outm = tail_mask(p0, T);
       const uint64_t M = st_mul[st][0];       // digest multiplier mix64(w) | 1
-      const bool final_word = (w == wend - 1);
       ev += __popc(E & outm);
       uint32_t bb = 0;  // bursts at max uncore: delivered x > theta
       if constexpr (bursts) {
@@ -482,7 +492,6 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
         }
         need_q |= (Lv[k] | pre_int[k]);
         B.carry = (B.carry & ~(1u << k)) | ((D >> 31) << k);
-        if (final_word) B.last |= ((D >> last_bit) & 1u) << k;
       }
       if (dec_row) dec_row += N;
       // model M stretch at min: once per sample, shared by the bundle
@@ -535,11 +544,31 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   }
 
   // ---------------- epilogue: publish, look back, correct ----------------
+  {
+  // the work coordinates, re-derived from the ticket rather than kept live
+  // across the scan (shadowing the names above)
+  const int32_t s = *(volatile int32_t*)&sh_work[0];
+  const int32_t bidx = *(volatile int32_t*)&sh_work[1];
+  const int32_t g = *(volatile int32_t*)&sh_work[2];
+  int32_t cfg[NB];
+#pragma unroll
+  for (int k = 0; k < NB; ++k) cfg[k] = __ldg(bundles + bidx * NB + k);
+  const int32_t c0 = cfg[0];
+  const int32_t t0 = wk.ts + (int32_t)(s * seg_len);
+  const int32_t t1 = (int32_t)((t0 + seg_len < T) ? t0 + seg_len : T);
+  const int32_t wt0 = t0 >> 5;
+  const int32_t wend = (t1 + 31) >> 5;
+  const int32_t ws = wk.ts >> 5;
+  const int64_t n = (int64_t)g * kTraces + tid;
+  const bool valid = n < N;
 #pragma unroll
   for (int k = 0; k < NB; ++k) {
     const int32_t c = cfg[k];
     if (!valid || c < 0) continue;
-    const uint32_t seen = (B.seen >> k) & 1u, last_min = (B.last >> k) & 1u;
+    // dec[t1-1] = bit 31 of the last word's fill when t1 % 32 == 0, i.e. for
+    // every segment but a trace's final one, whose status nobody reads (a
+    // resumed chunk boundary is a multiple of 32 by contract)
+    const uint32_t seen = (B.seen >> k) & 1u, last_min = (B.carry >> k) & 1u;
     uint32_t* status = wk.status + ((int64_t)c * nseg) * N + n;
     st_release(status + s * N, (wk.epoch << 3) | 1u | (seen << 1) | (last_min << 2));
   }
@@ -550,14 +579,21 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
     const bool seen = (B.seen >> k) & 1u;
     const BundleSmem& S = bs[k][tid];
     uint32_t* status = wk.status + ((int64_t)c * nseg) * N + n;
-    uint32_t cin = 0;  // true dec[t0-1]
+    const uint32_t hyp =
+        (s > 0) ? 1u : (wk.carry ? (__ldg(wk.carry + (int64_t)c * N + n) & 1u) : 0u);
+    uint32_t cin = hyp;  // true dec[t0-1] (segment 0: known)
     if (s > 0) {
+      // no action since the chunk start: the resume carry (read before this
+      // launch's finaliser may rewrite it: that waits for every segment)
+      cin = wk.carry ? (wk.carry[(int64_t)c * N + n] & 1u) : 0u;
       for (int64_t jj = s - 1; jj >= 0; --jj) {
         uint32_t v;
         while (((v = ld_acquire(status + jj * N)) >> 3) != wk.epoch) __nanosleep(32);
         if (v & 2u) { cin = (v >> 2) & 1u; break; }
       }
     }
+    if (wk.carry && s == nseg - 1)  // no successor reads it: republish as the chunk's final dec
+      st_release(status + s * N, (wk.epoch << 3) | 3u | ((seen ? (B.carry >> k) & 1u : cin) << 2));
     uint32_t hi, msr, mdec, mint, ch, bm, pb;
     if constexpr (kPack) {
       hi = B.cnt_a[k] & 0xFFFFu; msr = B.cnt_a[k] >> 16;
@@ -588,8 +624,8 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
       uint32_t* dec_out = wk.dec + (int64_t)c * wk.dec_cstride + n;
       const uint32_t fill = cin ? ~0u : 0u;
       const int32_t wlast = seen ? wt0 + S.wa : wend;
-      for (int32_t w = wt0; w < wlast; ++w) dec_out[w * N] = fill & tail_mask(w * 32, T);
-      if (seen) dec_out[(wt0 + S.wa) * N] = (S.dwa & ~S.pre_dec_a) | (fill & S.pre_dec_a);
+      for (int32_t w = wt0; w < wlast; ++w) dec_out[(w - ws) * N] = fill & tail_mask(w * 32, T);
+      if (seen) dec_out[(wt0 + S.wa - ws) * N] = (S.dwa & ~S.pre_dec_a) | (fill & S.pre_dec_a);
     }
     // segment sums -> per-(config, trace) accumulators (exact integer atomics)
     unsigned long long* acc = wk.acc + (int64_t)c * kAccFields * N + n;
@@ -627,8 +663,10 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
 #pragma unroll
         for (int q = 0; q < kAccFields; ++q) {
           a[q] = __ldcg(acc + q * N);
-          acc[q * N] = 0ULL;  // self-cleaning for the next replay
+          if (!wk.carry) acc[q * N] = 0ULL;  // self-cleaning for the next replay
         }
+        if (wk.carry)  // resume state: dec at the chunk's last interval (see above)
+          wk.carry[(int64_t)c * N + n] = (__ldcg(wk.status + ((int64_t)c * nseg + nseg - 1) * N + n) >> 2) & 1u;
         magus_summary sm_out;
         finalize_summary(plat, T, (int64_t)a[0], (int64_t)a[1], (int64_t)a[2], (int64_t)a[3],
                          (int64_t)a[4], (int64_t)a[5], a[6], a[7], a[8], a[9], (int64_t)a[10],
@@ -680,6 +718,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
       }
     }
     if (tid == 0) wk.arrive[(int64_t)c0 * ngroups + g] = 0;
+  }
   }
   if (tid == 0) {  // the last CTA of the launch re-arms the ticket counter
     __threadfence();

@@ -68,7 +68,20 @@ struct StreamWork {
   int64_t dec_cstride;           // nw * N
   uint64_t* totals;              // [C][18] or NULL
   const unsigned long long* mul; // [ceil(T/32)][2] {mix64(w) | 1, 0}: 16-B bulk-copy rows
+  // time-chunked replay (magus_replay_resume): the kernel works in global
+  // intervals [ts, T); buffer row r (TMA coordinate) is interval tb + r.
+  // Both are multiples of 32 (0, 0 for a one-shot replay).
+  int32_t tb, ts;
+  // resume state ([C][N] dec[t_start-1] bits, read at the start, rewritten by
+  // the finaliser once every segment of the (bundle, group) is in); NULL =
+  // one-shot replay.  In resume mode `acc` points into the caller's state and
+  // is kept (not self-cleaned).
+  uint32_t* carry;
 };
+// resume state layout: acc [C][kAccFields][N] u64, then carry [C][N] u32
+inline size_t resume_state_bytes(int64_t N, int32_t C) {
+  return 8 * (size_t)kAccFields * (size_t)C * (size_t)N + 4 * (size_t)C * (size_t)N;
+}
 
 // Host precompute (precompute.cpp); returns false + message on invalid input.
 bool validate_policy(const magus_policy& p, char* msg, size_t n);

@@ -131,3 +131,20 @@ def test_stretch_threshold_equals_literal_predicate():
             f = np.float32(thr)
             for x in (np.nextafter(f, np.float32(-np.inf)), f, np.nextafter(f, np.float32(np.inf))):
                 assert (x > f) == (float(x) * inv > 1.0)
+
+
+def test_resume_host_queries():
+    """magus_resume_halo = the rows before t_start that fix p_t and the Alg. 2
+    history (W + H - 1, rounded up to whole 32-step words); the state holds
+    12 u64 accumulators and one u32 carry per (config, trace)."""
+    import paper_conf_sc_zhengspl25_b200 as m
+    assert m.resume_halo([m.make_policy()]) == 32                      # 10 + 10 - 1 = 19
+    assert m.resume_halo([m.make_policy(W=16, H=10), m.make_policy(W=4, H=10)]) == 32  # 25
+    assert m.resume_halo([m.make_policy(W=33, H=32)]) == 64            # 64
+    assert m.resume_halo([m.make_policy(W=2, H=1)]) == 32              # 2 -> one word
+    nb = ctypes.c_size_t()
+    assert m._lib.magus_resume_state_bytes(1000, 3, ctypes.byref(nb)) == 0
+    assert nb.value == 3 * 1000 * (12 * 8 + 4)
+    assert m._lib.magus_resume_state_bytes(0, 3, ctypes.byref(nb)) != 0
+    with pytest.raises(m.MagusError):
+        m.resume_halo([m.make_policy(W=1)])
