@@ -34,6 +34,8 @@ WORKLOADS = {
     1: (1, 10_000, "default", 0, True, "cfg1: 1 trace x 10,000 intervals x 1 config (paper_default)"),
     2: (4096, 100_000, "default", 0, True, "cfg2: 4,096 traces x 100,000 intervals x 1 config (paper_default)"),
     3: (4096, 100_000, "sweep256", 0, False, "cfg3: 4,096 traces x 100,000 intervals x 256 configs (SWEEP256)"),
+    4: (65536, 1_000_000, "fleet64", 0, False,
+        "cfg4: 65,536 traces x 1,000,000 intervals x 64 configs (FLEET64), traces sharded over the GPUs"),
     5: (16384, 1_000_000, "default", 1, False,
         "cfg5: 16,384 adversarial traces x 1,000,000 intervals x 1 config (paper_default)"),
 }
@@ -127,7 +129,9 @@ def cpu_oracle_sample(cfg, T, pols_oracle, budget_s, kind, max_traces=None):
     seed = SEED_BASE + cfg
     # probe on a sample of the same shape class (time-major, ld = n): the
     # oracle reads each trace with stride ld, so a tiny probe under-estimates
-    probe_n = 64 if not max_traces else min(64, max_traces)
+    probe_n = max(1, min(64, int(2e7 / (T * len(pols_oracle)))))  # ~2 s of probe
+    if max_traces:
+        probe_n = min(probe_n, max_traces)
     xs = gen.gen_traces(seed, probe_n, T, kind=kind)
     t = time.perf_counter()
     oracle.replay(xs, pols_oracle)
@@ -170,10 +174,10 @@ def run_reference(args):
     import oracle
     pols = oracle_policies(policies_for(grid))
     seed = SEED_BASE + args.config
-    per_step = max(1, min(N, 4 if args.config != 5 else 1))
+    per_step = max(1, min(N, 4 if args.config not in (4, 5) else 1))
     xs = gen.gen_traces(seed, per_step, T, kind=kind)
-    if args.config == 3:
-        pols = pols[:16]  # bounded: 16 of the 256 configs per step
+    if args.config in (3, 4):
+        pols = pols[:16]  # bounded: 16 of the 256 / 64 configs per step
     for _ in range(args.warmup):
         oracle.replay(xs, pols)
     t = time.perf_counter()
@@ -400,6 +404,170 @@ def run_ours(args):
     return 0
 
 
+def run_fleet(args):
+    """Config 4: 65,536 traces x 10^6 intervals x FLEET64, traces sharded over
+    the GPUs (strong scaling: the fleet is fixed).  One GPU holds 262 GB of
+    traces only in time chunks: each step streams the fleet through HBM in
+    chunks of R intervals, generated on the device (untimed, SURVEY 8(d):
+    "trace generation is excluded") and replayed with magus_replay_resume
+    (timed: CUDA events around every replay call + the final all-reduce and
+    device-side choice).  The chunked replay is bit-identical to a one-shot
+    replay (tests/test_gpu_resume.py)."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sc_zhengspl25_b200 as magus
+    from paper_conf_sc_zhengspl25_b200 import dist as mdist
+
+    world, rank, local = dist_env()
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", init_method="env://")
+    dev = torch.device(f"cuda:{local}")
+    torch.cuda.set_device(dev)
+    stream = torch.cuda.current_stream(dev)
+    N_tot, T, grid, kind, _, desc = WORKLOADS[4]
+    if args.n_traces:
+        N_tot = args.n_traces
+    if args.n_steps:
+        T = args.n_steps
+    id0, N = mdist.shard(N_tot, world, rank)
+    pols = policies_for(grid)
+    C = len(pols)
+    seed = SEED_BASE + 4
+    ctx = magus.Context(device=local, stream=stream)
+    halo = magus.resume_halo(pols)
+    ld = (N + 3) // 4 * 4
+    R = args.chunk if args.chunk else min(T, (32 << 30) // (ld * 4))
+    R = max(halo, R // 32 * 32)
+    buf = torch.empty((halo + R, ld), dtype=torch.float32, device=dev)
+    gstate = ctx.gen_state(N)
+    state = ctx.resume_state(N, pols)
+    chunks = [(t, min(T, t + R)) for t in range(0, T, R)]
+    sweep_buf = None
+
+    def step(timed):
+        nonlocal sweep_buf
+        evs = []
+        out = None
+        for i, (t0, t1) in enumerate(chunks):
+            n = t1 - t0
+            if i > 0:  # the halo: the previous chunk's last rows
+                buf[:halo].copy_(buf[R:R + halo])
+            ctx.gen_traces_resume(seed, N, t0, n, gstate, buf[halo:halo + n], kind=kind, id0=id0)
+            a = torch.cuda.Event(enable_timing=True)
+            b = torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            if i == 0:
+                state.zero_()   # fresh accumulators for this pass
+                xs, tb = buf[halo:halo + n], 0
+            else:
+                xs, tb = buf[:halo + n], t0 - halo
+            last = i == len(chunks) - 1
+            out = ctx.replay_resume(xs, pols, state, t_base=tb, t_start=t0, n_traces=N, want_summary=False,
+                                    want_base=False, want_decisions=False, want_totals=last)
+            if last:
+                mdist.allreduce_totals(out.totals)
+                sweep_buf = ctx.sweep_best_async(out.totals, sweep_buf)
+            b.record(stream)
+            evs.append((a, b))
+        return evs, out
+
+    for _ in range(args.warmup):
+        step(False)
+    torch.cuda.synchronize()
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
+    ctx.set_option(magus.OPT_TIMING, 1)
+    ctx.reset_stats()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.mark()
+    all_evs = []
+    for _ in range(args.steps):
+        evs, out = step(True)
+        all_evs += evs
+    torch.cuda.synchronize()
+    clocks.mark()
+    best = ctx.sweep_result(sweep_buf)
+    if world > 1:
+        dist.barrier()
+    ms = sum(a.elapsed_time(b) for a, b in all_evs)
+    st = ctx.stats()
+    ctx.set_option(magus.OPT_TIMING, 0)
+    time.sleep(0.2)
+    clocks.stop()
+    kern_ms = st["main_ms_total"]
+    if world > 1:
+        t = torch.tensor([ms, kern_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms, kern_ms = float(t[0].item()), float(t[1].item())
+    ms_per_step = ms / args.steps
+    value = N_tot * T * C / (ms_per_step * 1e-3)
+    clk = clocks.summary()
+    sm_mhz = clk.get("sm_max_mhz") or 1965.0
+    alu_peak = 148 * 4 * 32 * sm_mhz * 1e6 / 1e9
+    alu_ach = 8.0 * N * T * C * args.steps / (kern_ms * 1e-3) / 1e9
+
+    # bounded oracle sample + parity of the chunked path at full T (untimed)
+    cpu = None
+    parity = None
+    if rank == 0 and not args.no_cpu_baseline:
+        import oracle
+        pol_o = oracle_policies(pols)[:16]
+        v, n_s, dt_s, ref = cpu_oracle_sample(4, T, pol_o, args.cpu_budget, kind, max_traces=64)
+        cpu = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"first {n_s} traces x {T} intervals x {len(pol_o)} configs of the fleet "
+                         f"({dt_s:.1f} s single-threaded)"}
+        if world == 1:
+            ld_s = (n_s + 3) // 4 * 4
+            sb = torch.empty((halo + R, ld_s), dtype=torch.float32, device=dev)
+            gs = ctx.gen_state(n_s)
+            rs = ctx.resume_state(n_s, pols[:16])
+            for i, (t0, t1) in enumerate(chunks):
+                n = t1 - t0
+                if i > 0:
+                    sb[:halo].copy_(sb[R:R + halo])
+                ctx.gen_traces_resume(seed, n_s, t0, n, gs, sb[halo:halo + n], kind=kind, id0=0)
+                xs, tb = (sb[halo:halo + n], 0) if i == 0 else (sb[:halo + n], t0 - halo)
+                r = ctx.replay_resume(xs, pols[:16], rs, t_base=tb, t_start=t0, n_traces=n_s,
+                                      want_summary=i == len(chunks) - 1, want_base=False, want_totals=False)
+            torch.cuda.synchronize()
+            got = r.summary_numpy()
+            parity = bool(all(np.array_equal(got[g], ref.summary[o]) for g, o in
+                              [("n_events", "n_events"), ("n_changes", "n_changes"), ("digest", "digest"),
+                               ("energy_j", "energy"), ("time_s", "time")]))
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": desc, "n_traces_total": N_tot, "n_traces_per_gpu": N, "n_steps": T,
+                       "n_configs": C, "decisions_emitted": False, "seed": hex(seed),
+                       "chunk_intervals": R, "chunks": len(chunks), "halo_rows": halo,
+                       "l2": f"chunks of {N * R * 4 / 1e9:.1f} GB > 126 MB L2 (no flush needed)",
+                       "timed": "replay calls + all-reduce + device choice; on-device generation of each "
+                                "chunk and the halo copy untimed (SURVEY 8(d))",
+                       "parallelism": f"traces sharded over {world} GPU(s); 1 NCCL all-reduce of int64 totals"},
+            "roofline": {"bound": "alu", "achieved": alu_ach, "peak": alu_peak, "unit": "Gop/s",
+                         "frac": alu_ach / alu_peak, "traffic": None,
+                         "peak_source": f"148 SMs x 128 lanes x {sm_mhz:.0f} MHz (B200_PROFILING.md unit counts)",
+                         "kernel": "stream_kernel", "kernel_ms": kern_ms / max(1, st["main_launches"]),
+                         "alg_ops_per_decision": 8},
+            "cpu_baseline": cpu,
+            "e2e": None, "e2e_note": "the fleet (262 GB) does not fit in host pinned memory; see cfg2 e2e",
+            "gpu_launches": int(st["launches_total"]), "clocks": clk,
+            "best_config": best[0], "feasible": best[2]}
+    if parity is not None:
+        line["parity_sample_ok"] = parity
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
 def run_bound(args):
     """NEXT f2: offline-optimal schedules (DP) on the workload, n_lambda weights.
     Unit: trace-sample x lambda.  ALU-bound on the fp64 pipe: ~12 fp64 ops per
@@ -482,6 +650,7 @@ def main():
     ap.add_argument("--step", type=int, default=1, help="ratio step of the gradual variant")
     ap.add_argument("--burst", type=float, default=0.0,
                     help="NEXT f1: Sec. 6.3 burst threshold (MB/s); > 0 enables the Jaccard counters")
+    ap.add_argument("--chunk", type=int, default=0, help="cfg4: intervals per time chunk (0 = fit ~32 GiB)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -493,6 +662,8 @@ def main():
         return run_bound(args)
     if args.impl == "reference":
         return run_reference(args)
+    if args.config == 4:
+        return run_fleet(args)
     return run_ours(args)
 
 

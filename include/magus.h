@@ -354,6 +354,16 @@ enum { MAGUS_GEN_MIX = 0, MAGUS_GEN_ADVERSARIAL = 1 };
 magus_status magus_gen_traces(magus_ctx ctx, uint64_t seed, int64_t id0,
                               int64_t n_traces, int64_t n_steps, int64_t ld,
                               int32_t kind, float* out);
+/* Time-chunked form (config 4 on one GPU: the traces never coexist in HBM):
+ * writes intervals [t0, t0 + n_rows) of the same traces to out rows
+ * 0..n_rows-1 (row stride ld).  `state` is a caller-owned DEVICE buffer of
+ * magus_gen_state_bytes(n_traces) bytes holding each trace's phase machine:
+ * t0 = 0 seeds it, later calls must continue at the previous t0 + n_rows.
+ * Concatenated chunks equal magus_gen_traces bit for bit.  Asynchronous. */
+magus_status magus_gen_state_bytes(int64_t n_traces, size_t* out);
+magus_status magus_gen_traces_resume(magus_ctx ctx, uint64_t seed, int64_t id0, int64_t n_traces,
+                                     int64_t t0, int64_t n_rows, int64_t ld, int32_t kind,
+                                     void* state, float* out);
 
 /* ---- diagnostics of the host precompute (no GPU needed) ----------------- */
 /* The stream kernel never divides: Alg. 1's "d = delta/L > tau_inc" becomes

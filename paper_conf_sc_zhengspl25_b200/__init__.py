@@ -112,6 +112,8 @@ _lib.magus_sweep_best_async.argtypes = [_vp, _vp, _i32, _vp]
 _lib.magus_totals_derive.argtypes = [_vp, _vp, ctypes.POINTER(Derived)]
 _lib.magus_sweep_best.argtypes = [_vp, _vp, _i32, ctypes.POINTER(_i32), ctypes.POINTER(Derived)]
 _lib.magus_gen_traces.argtypes = [_vp, _u64, _i64, _i64, _i64, _i64, _i32, _vp]
+_lib.magus_gen_traces_resume.argtypes = [_vp, _u64, _i64, _i64, _i64, _i64, _i64, _i32, _vp, _vp]
+_lib.magus_gen_state_bytes.argtypes = [_i64, ctypes.POINTER(ctypes.c_size_t)]
 _lib.magus_set_option.argtypes = [_vp, _i32, _i64]
 _lib.magus_policy_inspect.argtypes = [ctypes.POINTER(Policy), ctypes.POINTER(PolicyConsts)]
 _lib.magus_platform_inspect.argtypes = [ctypes.POINTER(Platform), ctypes.POINTER(PlatformConsts)]
@@ -137,7 +139,8 @@ EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_str
             "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
             "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host",
             "magus_replay_levels", "magus_offline_bound", "magus_sweep_best_async",
-            "magus_replay_resume", "magus_resume_state_bytes", "magus_resume_halo"]
+            "magus_replay_resume", "magus_resume_state_bytes", "magus_resume_halo",
+            "magus_gen_traces_resume", "magus_gen_state_bytes"]
 VARIANT_CLOSED_LOOP, VARIANT_GRADUAL = 1, 2
 
 
@@ -337,6 +340,21 @@ class Context:
         st = _lib.magus_gen_traces(self._h, seed & 0xFFFFFFFFFFFFFFFF, id0, n_traces, n_steps, ld, kind,
                                    _vp(out.data_ptr()))
         self._check(st, "gen_traces")
+        return out
+
+    def gen_state(self, n_traces: int):
+        """Device phase-machine state for gen_traces_resume."""
+        nb = ctypes.c_size_t()
+        if _lib.magus_gen_state_bytes(n_traces, ctypes.byref(nb)):
+            raise MagusError(1, "gen_state_bytes")
+        return self._torch.empty(((nb.value + 7) // 8,), dtype=self._torch.int64, device=f"cuda:{self.device}")
+
+    def gen_traces_resume(self, seed: int, n_traces: int, t0: int, n_rows: int, state, out, kind: int = GEN_MIX,
+                          id0: int = 0):
+        """Intervals [t0, t0 + n_rows) of the traces into out rows 0.. (out: [>= n_rows, ld])."""
+        st = _lib.magus_gen_traces_resume(self._h, seed & 0xFFFFFFFFFFFFFFFF, id0, n_traces, t0, n_rows,
+                                          out.stride(0), kind, _vp(state.data_ptr()), _vp(out.data_ptr()))
+        self._check(st, "gen_traces_resume")
         return out
 
     def replay(self, traces, policies, n_traces: int | None = None, want_summary: bool = True,

@@ -952,6 +952,25 @@ magus_status magus_gen_traces(magus_ctx ctx, uint64_t seed, int64_t id0, int64_t
   return MAGUS_OK;
 }
 
+magus_status magus_gen_state_bytes(int64_t n_traces, size_t* out) {
+  if (!out || n_traces < 1) return MAGUS_ERR_INVALID_ARG;
+  *out = gen_state_bytes(n_traces);
+  return MAGUS_OK;
+}
+
+magus_status magus_gen_traces_resume(magus_ctx ctx, uint64_t seed, int64_t id0, int64_t N, int64_t t0,
+                                     int64_t n_rows, int64_t ld, int32_t kind, void* state, float* out) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  if (!out || !state || (uintptr_t)state % 8 != 0 || N < 1 || n_rows < 1 || t0 < 0 || ld < N || id0 < 0 ||
+      (kind != MAGUS_GEN_MIX && kind != MAGUS_GEN_ADVERSARIAL))
+    return fail(ctx, MAGUS_ERR_INVALID_ARG, "bad gen_traces_resume arguments");
+  DeviceGuard dg(ctx->device);
+  if (launch_gen_resume(ctx->stream, seed, id0, N, t0, n_rows, ld, kind, state, out) < 0)
+    return cuda_fail(ctx, cudaGetLastError(), "gen kernel launch");
+  ctx->launches += 1;
+  return MAGUS_OK;
+}
+
 magus_status magus_get_stats(magus_ctx ctx, magus_stats* out) {
   if (!ctx || !out) return MAGUS_ERR_INVALID_ARG;
   DeviceGuard dg(ctx->device);

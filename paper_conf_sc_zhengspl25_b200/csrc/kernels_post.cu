@@ -164,6 +164,28 @@ int launch_digest_table(cudaStream_t s, unsigned long long* mul, int64_t nw) {
   return cudaGetLastError() == cudaSuccess ? 1 : -1;
 }
 
+// time-chunked generation: rows [t0, t0 + R) into out rows 0..R-1; the phase
+// machine of each trace is carried in `state` between chunks (t0 = 0 seeds it)
+__global__ void __launch_bounds__(128)
+gen_resume_kernel(uint64_t seed, int64_t id0, int64_t N, int64_t t0, int64_t R, int64_t ld,
+                  int32_t kind, mg_state* __restrict__ state, float* __restrict__ out) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= N) return;
+  mg_state g;
+  if (t0 == 0) mg_init(&g, seed, id0 + i, kind);
+  else g = state[i];
+  for (int64_t t = 0; t < R; ++t) out[t * ld + i] = (float)mg_step(&g);
+  state[i] = g;
+}
+
+int launch_gen_resume(cudaStream_t s, uint64_t seed, int64_t id0, int64_t N, int64_t t0, int64_t R,
+                      int64_t ld, int32_t kind, void* state, float* out) {
+  gen_resume_kernel<<<(unsigned)((N + 127) / 128), 128, 0, s>>>(seed, id0, N, t0, R, ld, kind,
+                                                                (mg_state*)state, out);
+  return cudaGetLastError() == cudaSuccess ? 1 : -1;
+}
+size_t gen_state_bytes(int64_t N) { return sizeof(mg_state) * (size_t)N; }
+
 int launch_gen(cudaStream_t s, uint64_t seed, int64_t id0, int64_t N, int64_t T, int64_t ld,
                int32_t kind, float* out) {
   gen_kernel<<<(unsigned)((N + 127) / 128), 128, 0, s>>>(seed, id0, N, T, ld, kind, out);

@@ -133,6 +133,9 @@ int launch_digest_table(cudaStream_t s, unsigned long long* mul, int64_t nw);
 
 int launch_gen(cudaStream_t s, uint64_t seed, int64_t id0, int64_t N, int64_t T, int64_t ld,
                int32_t kind, float* out);
+int launch_gen_resume(cudaStream_t s, uint64_t seed, int64_t id0, int64_t N, int64_t t0, int64_t R,
+                      int64_t ld, int32_t kind, void* state, float* out);
+size_t gen_state_bytes(int64_t N);
 
 // host-side derivation of fleet quantities (api.cu)
 void derive_totals(const DevPlatform& p, const uint64_t* w, magus_derived* out);

@@ -130,3 +130,17 @@ def test_resume_validation(ctx):
     gradual = [magus.make_policy(variant=magus.VARIANT_GRADUAL, step=1)]
     with pytest.raises(magus.MagusError):       # per-sample variants do not chunk
         ctx.replay_resume(buf, gradual, ctx.resume_state(N, gradual), t_base=0, t_start=0)
+
+
+@pytest.mark.parametrize("kind", [gen.KIND_MIX, gen.KIND_ADVERSARIAL])
+def test_gen_resume_matches_one_shot(ctx, kind):
+    """Chunked device generation == the host generator (and so == one shot)."""
+    N, T = 300, 2000
+    host = gen.gen_traces(gen.SEEDS[4] + kind, N, T, kind=kind, id0=77)
+    state = ctx.gen_state(N)
+    buf = torch.zeros((700, 304), dtype=torch.float32, device="cuda:0")
+    got = []
+    for t0, t1 in [(0, 5), (5, 700), (700, 1333), (1333, 2000)]:
+        ctx.gen_traces_resume(gen.SEEDS[4] + kind, N, t0, t1 - t0, state, buf, kind=kind, id0=77)
+        got.append(buf[: t1 - t0, :N].cpu().numpy().copy())
+    assert np.array_equal(np.concatenate(got), host)
