@@ -35,7 +35,13 @@ __device__ __forceinline__ uint64_t q_literal(float x, double invB) {
 // an fp64 add instead of the F2I conversion on the slow XU pipe.
 __device__ __forceinline__ uint64_t q_scaled(float x, double invB24) {
   double s24 = (double)x * invB24 - kQScale;
-  s24 = fmin(s24, kQCapScaled);
+  s24 = s24 < kQCapScaled ? s24 : kQCapScaled;  // never NaN here: x > xthr
+  return (uint64_t)__double_as_longlong(__dadd_rz(s24, 4503599627370496.0)) - 0x4330000000000000ULL;
+}
+// Same without the cap, for x <= x_stretch at ratio_max: s24 < (r_max/r_min)
+// * 2^24 <= 127 * 2^24 < 2^39 (ratio_max <= 127), so the cap never binds.
+__device__ __forceinline__ uint64_t q_scaled_nocap(float x, double invB24) {
+  const double s24 = (double)x * invB24 - kQScale;
   return (uint64_t)__double_as_longlong(__dadd_rz(s24, 4503599627370496.0)) - 0x4330000000000000ULL;
 }
 

@@ -62,16 +62,40 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 // try_wait with a suspend-time hint: a waiting warp is parked by the hardware
 // instead of re-issuing the probe (the producer otherwise burns ~20 % of the
 // SM's issue slots spinning on the empty barriers).
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+__device__ __forceinline__ void mbar_wait_s(uint32_t bar, uint32_t parity) {
   asm volatile(
       "{\n"
       ".reg .pred p;\n"
       "WAIT_%=:\n"
       "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n"
       "@!p bra WAIT_%=;\n"
-      "}\n" ::"r"(smem_u32(bar)),
+      "}\n" ::"r"(bar),
       "r"(parity), "r"(0x989680u)
       : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  mbar_wait_s(smem_u32(bar), parity);
+}
+__device__ __forceinline__ void mbar_arrive_s(uint32_t bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+// shared-window loads by 32-bit address (the generic->shared conversion of a
+// pointer costs an S2R + LEA each time the compiler rematerialises it)
+__device__ __forceinline__ float lds_f32(uint32_t a) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ unsigned long long lds_u64(uint32_t a) {
+  unsigned long long v;
+  asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ uint4 lds_v4(uint32_t a) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+  return v;
 }
 __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar,
                                             int32_t c0, int32_t c1) {
@@ -103,23 +127,13 @@ __device__ __forceinline__ void consumer_sync() {  // the 128 consumer threads o
 
 // ---- Alg. 2, bit-parallel: bit i of the result = (#events at positions
 // i-H .. i-1 >= k), positions < 0 coming from the previous word Ep. ----
-struct KMask {
-  uint32_t m[6];
-};
-__device__ __forceinline__ KMask make_kmask(int k) {
-  KMask r;
-#pragma unroll
-  for (int j = 0; j < 6; ++j) r.m[j] = ((k >> j) & 1) ? ~0u : 0u;
-  return r;
-}
-// count (bit-sliced, NB bits) >= k  <=>  no borrow out of count - k
+// count (bit-sliced, NB bits) >= k  <=>  no borrow out of count - k; km[j] =
+// all-ones where bit j of k is set (k < 2^NB always: k <= H + 1)
 template <int NB>
-__device__ __forceinline__ uint32_t ge_k(const uint32_t* c, const KMask& km) {
+__device__ __forceinline__ uint32_t ge_k(const uint32_t* c, const uint32_t* km) {
   uint32_t b = 0;
 #pragma unroll
-  for (int j = 0; j < NB; ++j) b = (~c[j] & km.m[j]) | (~c[j] & b) | (km.m[j] & b);  // maj
-#pragma unroll
-  for (int j = NB; j < 6; ++j) b |= km.m[j];  // k >= 2^NB: always borrows
+  for (int j = 0; j < NB; ++j) b = (~c[j] & km[j]) | (~c[j] & b) | (km[j] & b);  // maj: 1 LOP3
   return ~b;
 }
 __device__ __forceinline__ void fa(uint32_t a, uint32_t b, uint32_t c, uint32_t& s, uint32_t& cy) {
@@ -185,14 +199,15 @@ struct Window<0> {  // runtime H <= 32
 };
 
 // ---- Alg. 3 sample-and-hold: D_i = V at the last action <= i, else carry ----
-__device__ __forceinline__ uint32_t forward_fill(uint32_t A, uint32_t V, uint32_t carry_mask) {
-  uint32_t y = V & A, m = A;
-  y |= (y << 1) & ~m;  m |= m << 1;
-  y |= (y << 2) & ~m;  m |= m << 2;
-  y |= (y << 4) & ~m;  m |= m << 4;
-  y |= (y << 8) & ~m;  m |= m << 8;
-  y |= (y << 16) & ~m; m |= m << 16;
-  return y | (carry_mask & ~m);
+// A carry chain: a "set" (action to min, A & V) generates, a "reset" (action to
+// max, A & ~V) kills, every other position propagates.  The carries of
+// x + y + cin with x = ~(A & ~V), y = A & V are exactly that (x & y = set,
+// x ^ y = no action), so one 33-bit add replaces a 5-step log-depth fill.
+__device__ __forceinline__ uint32_t forward_fill(uint32_t A, uint32_t V, uint32_t cin) {
+  const uint32_t x = ~(A & ~V), y = A & V;
+  const uint64_t sum = (uint64_t)x + (uint64_t)y + (uint64_t)cin;
+  const uint32_t cin_bits = (uint32_t)sum ^ x ^ y;                // carry INTO bit i (bit 0: cin)
+  return __funnelshift_r(cin_bits, (uint32_t)(sum >> 32), 1);     // carry OUT of bit i
 }
 
 // w |= bit if a > b / a < b: one compare + one predicated LOP3 per bit
@@ -271,6 +286,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   // (tensor-copy destinations are 128-B aligned: one 128-B slot per stage)
   __shared__ __align__(128) unsigned long long st_mul[kStages][16];
   __shared__ BundleSmem bs[NB][kTraces];
+  __shared__ __align__(16) uint32_t s_km[NB][8];
 
   if (threadIdx.x == 0) {
     // launch-order work ticket -> (segment, bundle, group), segment-major so
@@ -371,16 +387,41 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   const bool bkeep = plat.burst_min_keeps != 0;     // B_min > theta: no burst is hidden
   const float xburst = plat.xburst;
   const bool want_dec = wk.dec != nullptr && valid;
-  uint32_t* dec_row = want_dec ? wk.dec + (wt0 - ws) * N + n : nullptr;  // + c * dec_cstride
+  // decision words of config cfg[0] (other bundle slots: + (cfg[k] - cfg[0]) * cstride)
+  uint32_t* dec_row = want_dec ? wk.dec + (int64_t)c0 * wk.dec_cstride + (int64_t)(wt0 - ws) * N + n
+                               : nullptr;
   double pd[W_T > 1 ? W_T - 1 : 1];  // previous word's last W-1 samples, widened
 #pragma unroll
   for (int k = 0; k < (W_T > 1 ? W_T - 1 : 1); ++k) pd[k] = 0.0;
 
+  // Alg. 2 threshold masks of each bundle slot (km[j] = all-ones iff bit j of
+  // k is set), read back with one 16-B shared load per word and slot
+  constexpr int kNBits = Window<H_T>::NBITS;
+  static_assert(kNBits <= 8, "km table");
+  if (tid < NB * kNBits) {
+    const int kslot = tid / kNBits, j = tid % kNBits;
+    int32_t kv = 0x3F;
+#pragma unroll
+    for (int k = 0; k < NB; ++k)
+      if (k == kslot) kv = kk[k];
+    s_km[kslot][j] = ((kv >> j) & 1) ? ~0u : 0u;
+  }
+  consumer_sync();
+  const uint32_t km_s = smem_u32(&s_km[0][0]);
+  const uint32_t full_s = smem_u32(&full_bar[0]), empty_s = smem_u32(&empty_bar[0]);
+  const uint32_t sm_s = smem_u32(sm) + 4u * (uint32_t)tid;  // this thread's column
+  const uint32_t mul_s = smem_u32(&st_mul[0][0]);
+  // words of the trace's last (partial) word and of the warm-up
+  const int32_t Ti = (int32_t)T;
+  const int32_t w_tail = (Ti - 1) >> 5;
+  const uint32_t tail_m = (Ti & 31) ? ((1u << (Ti & 31)) - 1u) : ~0u;
+
   int st = 0, pst = kStages - 1;
   uint32_t ph = 0;
   for (int32_t j = 0; j < nwords; ++j) {
-    mbar_wait(&full_bar[st], ph);
+    mbar_wait_s(full_s + 8u * (uint32_t)st, ph);
     const float* cur = sm + st * kStageFloats + tid;
+    const uint32_t cur_s = sm_s + (uint32_t)(st * kStageFloats * 4);
     const int32_t w = w_first + j;
     const int32_t p0 = w * 32;
 
@@ -416,15 +457,22 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
         wmax = fmaxf(wmax, xi);
       }
     }
-    // warp-uniform word constants (kept in uniform registers by the compiler)
-    const uint32_t warm = (p0 >= W) ? 0u : ((W - p0) >= 32 ? ~0u : ((1u << (W - p0)) - 1u));
+    // warm-up rounds t < W (Alg. 3 runs from t = W): words 0 and (W = 33) 1 only
+    uint32_t warm;
+    if constexpr (W_T > 0) {
+      constexpr uint32_t kWarm0 = W_T >= 32 ? ~0u : ((1u << W_T) - 1u);
+      constexpr uint32_t kWarm1 = W_T > 32 ? ((1u << (W_T - 32)) - 1u) : 0u;
+      warm = (p0 == 0) ? kWarm0 : ((W_T > 32 && p0 == 32) ? kWarm1 : 0u);
+    } else {
+      warm = (p0 >= W) ? 0u : ((W - p0) >= 32 ? ~0u : ((1u << (W - p0)) - 1u));
+    }
     const uint32_t incv = incw & ~warm;          // p = +1
     const uint32_t decv = decw & ~warm & ~incv;  // p = -1 (line 4 before line 6)
     const uint32_t E = incv | decv;              // uncore_tune_ls.push_back(1)
 
     if (w >= wt0) {
-      const uint32_t outm = tail_mask(p0, T);
-      const uint64_t M = st_mul[st][0];       // digest multiplier mix64(w) | 1
+      const uint32_t outm = (w == w_tail) ? tail_m : ~0u;
+      const uint64_t M = lds_u64(mul_s + 128u * (uint32_t)st);  // digest multiplier mix64(w) | 1
       ev += __popc(E & outm);
       uint32_t bb = 0;  // bursts at max uncore: delivered x > theta
       if constexpr (bursts) {
@@ -434,18 +482,27 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
         bbase += __popc(bb);
       }
       // Alg. 2 (l.9): the count of the H previous events, shared by the bundle
-      uint32_t cnt[Window<H_T>::NBITS];
+      uint32_t cnt[kNBits];
       Window<H_T>::count(E, Eprev, H, cnt);
       uint32_t Lv[NB], pre_int[NB];
-      uint32_t need_q = 0;
+      uint32_t need_q = 0, pre_any = 0;
 #pragma unroll
       for (int k = 0; k < NB; ++k) {
         const uint32_t ck = (B.carry >> k) & 1u;
-        const uint32_t HI = ge_k<Window<H_T>::NBITS>(cnt, make_kmask(kk[k])) & ~warm;
+        uint32_t km[kNBits];
+        {
+          const uint4 a = lds_v4(km_s + 32u * k);
+          km[0] = a.x; km[1] = a.y; km[2] = a.z; km[3] = a.w;
+          if constexpr (kNBits > 4) {
+            const uint4 b2 = lds_v4(km_s + 32u * k + 16u);
+            km[4] = b2.x; km[5] = b2.y;
+          }
+        }
+        const uint32_t HI = ge_k<kNBits>(cnt, km) & ~warm;
         const uint32_t act = HI | E;                 // tune_uncore_freq calls (l.11/19/25)
         const uint32_t A = act | warm;               // positions that set the frequency
         const uint32_t V = decv & ~HI;               // ... to min (l.25)
-        const uint32_t D = forward_fill(A, V, ck ? ~0u : 0u);
+        const uint32_t D = forward_fill(A, V, ck);
         Lv[k] = (D << 1) | ck;                       // interval level = dec[t-1]
         uint32_t chm = (D ^ Lv[k]) & outm;
         if (p0 == 0) chm &= ~1u;
@@ -482,7 +539,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
           }
           bs[k][tid].pdig += (unsigned long long)pre_dec * M;
         } else if (want_dec && cfg[k] >= 0) {
-          dec_row[(int64_t)cfg[k] * wk.dec_cstride] = Dout;
+          dec_row[(int64_t)(cfg[k] - c0) * wk.dec_cstride] = Dout;
         }
         if constexpr (bursts) {  // kept unless the interval ran at a level whose capacity hides it
           const uint32_t kept = bkeep ? bb : (bb & ~Lv[k]);
@@ -490,43 +547,62 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
           if constexpr (kPack) B.cnt_f[k] += (uint32_t)__popc(kept) | ((uint32_t)__popc(pb) << 16);
           else { B.cnt_f[k] += __popc(kept); B.cnt_g[k] += __popc(pb); }
         }
-        need_q |= (Lv[k] | pre_int[k]);
+        need_q |= Lv[k];
+        pre_any |= pre_int[k];
         B.carry = (B.carry & ~(1u << k)) | ((D >> 31) << k);
       }
-      if (dec_row) dec_row += N;
+      if (want_dec) dec_row += N;
       // model M stretch at min: once per sample, shared by the bundle
-      uint32_t mq = smin & need_q & outm;
-      while (mq) {  // order-free integer sums; two independent chains per trip
-        const int i1 = 31 - __clz(mq);
-        const uint32_t m1 = 1u << i1;
-        mq ^= m1;
-        const int i2 = mq ? 31 - __clz(mq) : i1;
-        const uint32_t m2 = mq ? 1u << i2 : 0u;
-        mq ^= m2;
-        const unsigned long long q1 = q_scaled(cur[i1 * kTraces], invB24_min);
-        const unsigned long long q2 = m2 ? q_scaled(cur[i2 * kTraces], invB24_min) : 0ULL;
-#pragma unroll
-        for (int k = 0; k < NB; ++k) {
-          if (Lv[k] & m1) B.qmin[k] += q1;
-          if (pre_int[k] & m1) B.pqmin[k] += q1;
-          if (Lv[k] & m2) B.qmin[k] += q2;
-          if (pre_int[k] & m2) B.pqmin[k] += q2;
-        }
-      }
-      if (wmax > xthr_max) {  // some sample exceeds even the capacity at max (rare)
-        uint32_t mx = smin & outm;  // x > xthr_max implies x > xthr_min
-        while (mx) {
-          const int i = 31 - __clz(mx);
-          const uint32_t m1 = 1u << i;
-          mx ^= m1;
-          const float xi = cur[i * kTraces];
-          if (xi > xthr_max) {
-            const unsigned long long q = q_scaled(xi, invB24_max);
-            qbase += q;
+      if (wmax <= xthr_max && pre_any == 0) {
+        // common case: no sample above the capacity at max (so s24 < 127 * 2^24
+        // needs no cap: ratio_max <= 127), no carry-dependent prefix
+        uint32_t mq = smin & need_q & outm;
+        while (mq) {  // order-free integer sums; two independent chains per trip
+          const int i1 = 31 - __clz(mq);
+          mq ^= 1u << i1;
+          const int i2 = mq ? 31 - __clz(mq) : i1;
+          const uint32_t m2 = mq ? 1u << i2 : 0u;
+          mq ^= m2;
+          const unsigned long long q1 = q_scaled_nocap(lds_f32(cur_s + 512u * i1), invB24_min);
+          const unsigned long long q2 = q_scaled_nocap(lds_f32(cur_s + 512u * i2), invB24_min);
+          if constexpr (NB == 1) {
+            B.qmin[0] += q1 + (m2 ? q2 : 0ULL);
+          } else {
 #pragma unroll
             for (int k = 0; k < NB; ++k) {
-              if (!(Lv[k] & m1)) bs[k][tid].qmax += q;
-              if (pre_int[k] & m1) bs[k][tid].pqmax += q;
+              if ((Lv[k] >> i1) & 1u) B.qmin[k] += q1;
+              if (Lv[k] & m2) B.qmin[k] += q2;
+            }
+          }
+        }
+      } else {
+        uint32_t mq = smin & (need_q | pre_any) & outm;
+        while (mq) {
+          const int i1 = 31 - __clz(mq);
+          const uint32_t m1 = 1u << i1;
+          mq ^= m1;
+          const unsigned long long q1 = q_scaled(lds_f32(cur_s + 512u * i1), invB24_min);
+#pragma unroll
+          for (int k = 0; k < NB; ++k) {
+            if (Lv[k] & m1) B.qmin[k] += q1;
+            if (pre_int[k] & m1) B.pqmin[k] += q1;
+          }
+        }
+        if (wmax > xthr_max) {  // some sample exceeds even the capacity at max (rare)
+          uint32_t mx = smin & outm;  // x > xthr_max implies x > xthr_min
+          while (mx) {
+            const int i = 31 - __clz(mx);
+            const uint32_t m1 = 1u << i;
+            mx ^= m1;
+            const float xi = lds_f32(cur_s + 512u * i);
+            if (xi > xthr_max) {
+              const unsigned long long q = q_scaled(xi, invB24_max);
+              qbase += q;
+#pragma unroll
+              for (int k = 0; k < NB; ++k) {
+                if (!(Lv[k] & m1)) bs[k][tid].qmax += q;
+                if (pre_int[k] & m1) bs[k][tid].pqmax += q;
+              }
             }
           }
         }
@@ -535,9 +611,9 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
     Eprev = E;
     __syncwarp();
     if constexpr (W_T > 0) {
-      if (lane == 0) mbar_arrive(&empty_bar[st]);                      // word read: free
+      if (lane == 0) mbar_arrive_s(empty_s + 8u * (uint32_t)st);          // word read: free
     } else {
-      if (j >= 1 && lane == 0) mbar_arrive(&empty_bar[pst]);           // lag read: free
+      if (j >= 1 && lane == 0) mbar_arrive_s(empty_s + 8u * (uint32_t)pst);  // lag read: free
     }
     pst = st;
     if (++st == kStages) { st = 0; ph ^= 1u; }
