@@ -1,6 +1,7 @@
 """C-ABI surface checks that need no GPU: the library loads, exports every
 function include/magus.h declares, and its host-only calls behave."""
 import ctypes
+import functools
 import os
 import re
 
@@ -72,6 +73,12 @@ def test_null_context_is_rejected():
     assert m._lib.magus_status_string(m.ERR_NO_FEASIBLE) == b"no feasible config"
 
 
+@functools.lru_cache(maxsize=2)
+def _sass(tool: str, lib: str, mtime: float) -> str:
+    import subprocess
+    return subprocess.run([tool, "-sass", lib], capture_output=True, text=True, check=True).stdout
+
+
 def _consumer_loop_local_ops(sass: str):
     """Local-memory (spill) instructions inside the consumer's word loop: the
     largest backward branch whose target sits just before an mbarrier wait."""
@@ -101,7 +108,6 @@ def test_hot_kernels_do_not_spill_in_the_word_loop(inst, budget):
     reload at most two loop-invariant words per 32-step word (~1000
     instructions).  A few bytes spilled around the loop are harmless."""
     import shutil
-    import subprocess
     log = open(os.path.join(ROOT, "paper_conf_sc_zhengspl25_b200", "build", "ptxas.log")).read()
     blocks = [b for b in re.split(r"Compiling entry function", log) if "stream_kernel" + inst in b]
     assert blocks, f"stream_kernel{inst} missing from the build"
@@ -111,7 +117,7 @@ def test_hot_kernels_do_not_spill_in_the_word_loop(inst, budget):
     if not os.path.exists(tool) and not shutil.which("cuobjdump"):
         pytest.skip("cuobjdump unavailable")
     lib = os.path.join(ROOT, "paper_conf_sc_zhengspl25_b200", "libmagus.so")
-    out = subprocess.run([tool, "-sass", lib], capture_output=True, text=True, check=True).stdout
+    out = _sass(tool, lib, os.path.getmtime(lib))
     fn = [p for p in out.split("Function : ") if "stream_kernel" + inst in p.split("\n")[0]]
     assert fn
     size, local = _consumer_loop_local_ops(fn[0])
