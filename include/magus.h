@@ -391,7 +391,10 @@ enum {
   MAGUS_OPT_KERNEL = 0,       /* 0 auto, 1 reference (per-sample), 2 stream  */
   MAGUS_OPT_SEGMENTS = 1,     /* 0 auto, else the number of time segments    */
   MAGUS_OPT_TIMING = 2,       /* 1: record CUDA events around the main kernel */
-  MAGUS_OPT_WAVES = 3,        /* target waves for auto segmentation (def. 4) */
+  MAGUS_OPT_WAVES = 3,        /* auto segmentation: 0 (default) = wave model
+                                 (segment count minimising the modelled
+                                 rounds x segment length), else aim at this
+                                 many waves of CTAs                          */
   MAGUS_OPT_BUNDLE = 4        /* configs per thread sharing Alg. 1/2 work:
                                  0 auto, or force 1, 2 or 4                  */
 };

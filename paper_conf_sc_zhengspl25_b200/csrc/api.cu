@@ -25,7 +25,7 @@ struct magus_ctx_s {
   std::string err;
   int sms = 148;
   // options
-  int64_t opt_kernel = 0, opt_segments = 0, opt_timing = 0, opt_waves = 4;
+  int64_t opt_kernel = 0, opt_segments = 0, opt_timing = 0, opt_waves = 0;
   // device scratch
   void* scratch = nullptr;
   size_t scratch_bytes = 0;
@@ -498,7 +498,7 @@ magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value) {
       ctx->opt_bundle = value;
       return MAGUS_OK;
     case MAGUS_OPT_WAVES:
-      if (value < 1 || value > 64) return fail(ctx, MAGUS_ERR_INVALID_ARG, "waves not in [1, 64]");
+      if (value < 0 || value > 64) return fail(ctx, MAGUS_ERR_INVALID_ARG, "waves not in [0, 64]");
       ctx->opt_waves = value;
       return MAGUS_OK;
   }
@@ -554,8 +554,36 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
   int64_t nseg = 1, seg_len = ((Tr + 31) / 32) * 32;
   if (kernel == 2) {
     const int64_t ngroups = (N + 127) / 128;
+    bool packed = false;  // NB > 1 packs per-segment counters in 16 bits
+    for (auto& g : ctx->groups) packed = packed || g.NB > 1;
     if (ctx->opt_segments > 0) {
       nseg = ctx->opt_segments;
+    } else if (ctx->opt_waves == 0) {
+      // Wave model: the launches of the W groups run back to back and every
+      // CTA of a launch streams one segment, so a launch takes
+      // ceil(CTAs / resident slots) rounds of (segment + halo + fixed epilogue)
+      // steps.  Pick the segment count with the smallest modelled total
+      // (fewer segments on ties: less halo re-read and look-back).
+      const int64_t words = (Tr + 31) / 32;
+      const int64_t lo = packed ? (words * 32 + 65503) / 65504 : 1;
+      const int64_t hi = std::max<int64_t>(lo, std::min<int64_t>(words / 16, 4096));  // >= 512 steps
+      double best_cost = 0.0;
+      nseg = lo;
+      for (int64_t cand = lo; cand <= hi; ++cand) {
+        const int64_t len = ((Tr + cand - 1) / cand + 31) / 32 * 32;
+        if ((Tr + len - 1) / len != cand) continue;  // not realisable with 32-step segments
+        double cost = 0.0;
+        for (auto& g : ctx->groups) {
+          const int64_t slots = (int64_t)ctx->sms * std::max(1, ctas_per_sm(ctx, g.W, g.H, g.NB));
+          const int64_t ctas = ngroups * g.nbund * cand;
+          const int64_t halo = cand > 1 ? ((g.W + g.H - 1 + 31) / 32) * 32 : 0;
+          cost += (double)((ctas + slots - 1) / slots) * (double)(len + halo + 96);
+        }
+        if (cand == lo || cost < best_cost * 0.999) {
+          best_cost = cost;
+          nseg = cand;
+        }
+      }
     } else {
       int per_sm = 1 << 30;
       int64_t nbund = 0;
@@ -568,8 +596,6 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
       nseg = std::max<int64_t>(1, (slots + ngroups * nbund - 1) / (ngroups * nbund));
     }
     seg_len = ((Tr + nseg - 1) / nseg + 31) / 32 * 32;
-    bool packed = false;  // NB > 1 packs per-segment counters in 16 bits
-    for (auto& g : ctx->groups) packed = packed || g.NB > 1;
     if (packed && seg_len > 65504) seg_len = 65504;
     const int64_t min_len = 512;  // keeps the halo re-read below ~6 %
     if (ctx->opt_segments == 0 && seg_len < min_len) seg_len = std::min<int64_t>(min_len, ((Tr + 31) / 32) * 32);
