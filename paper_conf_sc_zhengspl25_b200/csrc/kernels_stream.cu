@@ -388,8 +388,11 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   const float xburst = plat.xburst;
   const bool want_dec = wk.dec != nullptr && valid;
   // decision words of config cfg[0] (other bundle slots: + (cfg[k] - cfg[0]) * cstride)
-  uint32_t* dec_row = want_dec ? wk.dec + (int64_t)c0 * wk.dec_cstride + (int64_t)(wt0 - ws) * N + n
-                               : nullptr;
+  // (an integer address, advanced every word whether or not it is used)
+  uint64_t dec_row = want_dec ? reinterpret_cast<uint64_t>(wk.dec + (int64_t)c0 * wk.dec_cstride +
+                                                           (int64_t)(wt0 - ws) * N + n)
+                              : 0;
+  const uint64_t dec_step = 4ull * (uint64_t)N;
   double pd[W_T > 1 ? W_T - 1 : 1];  // previous word's last W-1 samples, widened
 #pragma unroll
   for (int k = 0; k < (W_T > 1 ? W_T - 1 : 1); ++k) pd[k] = 0.0;
@@ -416,9 +419,9 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   const int32_t w_tail = (Ti - 1) >> 5;
   const uint32_t tail_m = (Ti & 31) ? ((1u << (Ti & 31)) - 1u) : ~0u;
 
-  int st = 0, pst = kStages - 1;
-  uint32_t ph = 0;
-  for (int32_t j = 0; j < nwords; ++j) {
+  // one 32-step word of the scan; st / pst = stage of this / the previous word
+  auto word = [&](const int st, const int pst, const uint32_t ph, const int32_t j)
+                  __attribute__((always_inline)) {
     mbar_wait_s(full_s + 8u * (uint32_t)st, ph);
     const float* cur = sm + st * kStageFloats + tid;
     const uint32_t cur_s = sm_s + (uint32_t)(st * kStageFloats * 4);
@@ -504,8 +507,8 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
         const uint32_t V = decv & ~HI;               // ... to min (l.25)
         const uint32_t D = forward_fill(A, V, ck);
         Lv[k] = (D << 1) | ck;                       // interval level = dec[t-1]
-        uint32_t chm = (D ^ Lv[k]) & outm;
-        if (p0 == 0) chm &= ~1u;
+        // (t = 0: D_0 = 0 (warm-up) and the carry is max, so bit 0 is clear)
+        const uint32_t chm = (D ^ Lv[k]) & outm;
         const uint32_t Dout = D & outm;
         if constexpr (kPack) {
           B.cnt_a[k] += (uint32_t)__popc(HI & outm) | ((uint32_t)__popc(act & outm) << 16);
@@ -539,7 +542,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
           }
           bs[k][tid].pdig += (unsigned long long)pre_dec * M;
         } else if (want_dec && cfg[k] >= 0) {
-          dec_row[(int64_t)(cfg[k] - c0) * wk.dec_cstride] = Dout;
+          reinterpret_cast<uint32_t*>(dec_row)[(int64_t)(cfg[k] - c0) * wk.dec_cstride] = Dout;
         }
         if constexpr (bursts) {  // kept unless the interval ran at a level whose capacity hides it
           const uint32_t kept = bkeep ? bb : (bb & ~Lv[k]);
@@ -551,7 +554,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
         pre_any |= pre_int[k];
         B.carry = (B.carry & ~(1u << k)) | ((D >> 31) << k);
       }
-      if (want_dec) dec_row += N;
+      dec_row += dec_step;
       // model M stretch at min: once per sample, shared by the bundle
       if (wmax <= xthr_max && pre_any == 0) {
         // common case: no sample above the capacity at max (so s24 < 127 * 2^24
@@ -615,8 +618,27 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
     } else {
       if (j >= 1 && lane == 0) mbar_arrive_s(empty_s + 8u * (uint32_t)pst);  // lag read: free
     }
-    pst = st;
-    if (++st == kStages) { st = 0; ph ^= 1u; }
+  };
+  if constexpr (NB == 1) {
+    // one config per thread: the ring is unrolled by its depth, so the stage
+    // (and with it every shared address of the word) is a compile-time
+    // constant (the 4-config body is too large to triple: I-cache)
+    uint32_t ph = 0;
+    for (int32_t j0 = 0; j0 < nwords; j0 += kStages, ph ^= 1u) {
+#pragma unroll
+      for (int st = 0; st < kStages; ++st) {
+        if (j0 + st >= nwords) break;
+        word(st, st == 0 ? kStages - 1 : st - 1, ph, j0 + st);
+      }
+    }
+  } else {
+    int st = 0, pst = kStages - 1;
+    uint32_t ph = 0;
+    for (int32_t j = 0; j < nwords; ++j) {
+      word(st, pst, ph, j);
+      pst = st;
+      if (++st == kStages) { st = 0; ph ^= 1u; }
+    }
   }
 
   // ---------------- epilogue: publish, look back, correct ----------------
