@@ -1,0 +1,18 @@
+set -x
+O=gpurun_out/r1
+mkdir -p $O
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.limit --format=csv > $O/gpu.txt 2>&1
+python bench.py > $O/bench_cfg2.json 2> $O/bench_cfg2.err
+python bench.py --config 3 --steps 20 --warmup 3 > $O/bench_cfg3.json 2> $O/bench_cfg3.err
+python bench.py --config 5 --steps 20 --warmup 3 > $O/bench_cfg5.json 2> $O/bench_cfg5.err
+python bench.py --config 4 --steps 2 --warmup 3 > $O/bench_cfg4.json 2> $O/bench_cfg4.err
+python bench.py --burst 12000 --steps 300 --no-cpu-baseline --no-e2e > $O/bench_cfg2_f1.json 2> $O/bench_cfg2_f1.err
+python bench.py --bound 8 --steps 3 --warmup 3 > $O/bench_cfg2_f2.json 2> $O/bench_cfg2_f2.err
+python bench.py --bound 4 --full-grid --steps 2 --warmup 3 > $O/bench_cfg2_f2full.json 2> $O/bench_cfg2_f2full.err
+python bench.py --variant 1 --steps 10 --warmup 3 --no-cpu-baseline --no-e2e > $O/bench_cfg2_f3.json 2> $O/bench_cfg2_f3.err
+python bench.py --variant 2 --step 2 --steps 10 --warmup 3 --no-cpu-baseline --no-e2e > $O/bench_cfg2_f4.json 2> $O/bench_cfg2_f4.err
+python bench.py --impl reference --steps 3 --warmup 3 > $O/bench_ref_cfg2.json 2> $O/bench_ref_cfg2.err
+ncu --set full --import-source on --clock-control none -k regex:stream_kernel --launch-skip 3 -c 1 -o $O/prof_cfg2 python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > $O/ncu_cfg2.log 2>&1
+ncu --set full --import-source on --clock-control none -k regex:stream_kernel --launch-skip 12 -c 1 -o $O/prof_cfg3 python bench.py --config 3 --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > $O/ncu_cfg3.log 2>&1
+ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_cfg2.csv python bench.py --steps 20 --warmup 3 --no-cpu-baseline --no-e2e > /dev/null 2>&1
+ls -la $O
