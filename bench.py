@@ -115,6 +115,24 @@ class ClockSampler:
         return out
 
 
+def setup_dist(world: int, local: int) -> int:
+    """One process per GPU; returns this rank's CUDA device index.  The
+    backend is NCCL; MAGUS_DIST_BACKEND=gloo (with several ranks sharing a
+    GPU, device = local rank mod the GPU count) exercises the multi-rank path
+    of this script on a single-GPU box."""
+    import torch
+    import torch.distributed as dist
+    devidx = local % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(devidx)
+    if world > 1:
+        dist.init_process_group(os.environ.get("MAGUS_DIST_BACKEND", "nccl"), init_method="env://")
+    return devidx
+
+
+def dist_backend(world: int) -> str:
+    return "none" if world == 1 else os.environ.get("MAGUS_DIST_BACKEND", "nccl")
+
+
 def dist_env():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -206,11 +224,8 @@ def run_ours(args):
     world, rank, local = dist_env()
     if world != args.gpus:
         print(f"warning: --gpus {args.gpus} but WORLD_SIZE {world}", file=sys.stderr)
-    if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", init_method="env://")
+    local = setup_dist(world, local)
     dev = torch.device(f"cuda:{local}")
-    torch.cuda.set_device(dev)
     stream = torch.cuda.current_stream(dev)
 
     N, T, grid, kind, want_dec, desc = WORKLOADS[args.config]
@@ -381,7 +396,7 @@ def run_ours(args):
             "config": {"workload": desc, "n_traces_per_gpu": N, "n_traces_total": N * world, "n_steps": T,
                        "n_configs": C, "decisions_emitted": want_dec, "seed": hex(seed),
                        "l2": f"inputs {N * T * 4 / 1e9:.2f} GB per GPU > 126 MB L2 (no flush needed)",
-                       "parallelism": f"traces sharded over {world} GPU(s); 1 NCCL all-reduce of int64 totals",
+                       "parallelism": f"traces sharded over {world} GPU(s); 1 all-reduce of int64 totals ({dist_backend(world)})",
                        "segments": st["last_segments"], "kernel": "stream" if st["last_kernel"] == 2 else "reference",
                        "variant": args.variant, "step": args.step if args.variant & 2 else 0},
             "roofline": roof,
@@ -420,11 +435,8 @@ def run_fleet(args):
     from paper_conf_sc_zhengspl25_b200 import dist as mdist
 
     world, rank, local = dist_env()
-    if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", init_method="env://")
+    local = setup_dist(world, local)
     dev = torch.device(f"cuda:{local}")
-    torch.cuda.set_device(dev)
     stream = torch.cuda.current_stream(dev)
     N_tot, T, grid, kind, _, desc = WORKLOADS[4]
     if args.n_traces:
@@ -548,7 +560,7 @@ def run_fleet(args):
                        "l2": f"chunks of {N * R * 4 / 1e9:.1f} GB > 126 MB L2 (no flush needed)",
                        "timed": "replay calls + all-reduce + device choice; on-device generation of each "
                                 "chunk and the halo copy untimed (SURVEY 8(d))",
-                       "parallelism": f"traces sharded over {world} GPU(s); 1 NCCL all-reduce of int64 totals"},
+                       "parallelism": f"traces sharded over {world} GPU(s); 1 all-reduce of int64 totals ({dist_backend(world)})"},
             "roofline": {"bound": "alu", "achieved": alu_ach, "peak": alu_peak, "unit": "Gop/s",
                          "frac": alu_ach / alu_peak, "traffic": None,
                          "peak_source": f"148 SMs x 128 lanes x {sm_mhz:.0f} MHz (B200_PROFILING.md unit counts)",
