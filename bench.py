@@ -397,7 +397,7 @@ def run_ours(args):
                        "n_configs": C, "decisions_emitted": want_dec, "seed": hex(seed),
                        "l2": f"inputs {N * T * 4 / 1e9:.2f} GB per GPU > 126 MB L2 (no flush needed)",
                        "parallelism": f"traces sharded over {world} GPU(s); 1 all-reduce of int64 totals ({dist_backend(world)})",
-                       "segments": st["last_segments"], "kernel": "stream" if st["last_kernel"] == 2 else "reference",
+                       "segments": st["last_segments"], "kernel": {1: "reference", 2: "stream", 3: "sequential"}.get(st["last_kernel"], "?"),
                        "variant": args.variant, "step": args.step if args.variant & 2 else 0},
             "roofline": roof,
             "cpu_baseline": cpu, "e2e": e2e,

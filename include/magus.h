@@ -388,7 +388,11 @@ magus_status magus_platform_inspect(const magus_platform* p, magus_platform_cons
 
 /* ---- options, instrumentation ------------------------------------------ */
 enum {
-  MAGUS_OPT_KERNEL = 0,       /* 0 auto, 1 reference (per-sample), 2 stream  */
+  MAGUS_OPT_KERNEL = 0,       /* 0 auto, 1 reference (per-sample, the printed
+                                 divisions), 2 stream, 3 sequential (per-sample,
+                                 latency-optimised: f3/f4 and level output;
+                                 the auto choice when the stream kernel cannot
+                                 run)                                        */
   MAGUS_OPT_SEGMENTS = 1,     /* 0 auto, else the number of time segments    */
   MAGUS_OPT_TIMING = 2,       /* 1: record CUDA events around the main kernel */
   MAGUS_OPT_WAVES = 3,        /* auto segmentation: 0 (default) = wave model
@@ -405,7 +409,7 @@ typedef struct {
   int64_t main_launches;      /* replay-kernel launches timed (OPT_TIMING)   */
   double  main_ms_total;      /* summed CUDA-event time of those launches    */
   int64_t last_segments;      /* time segments used by the last replay       */
-  int64_t last_kernel;        /* 1 reference, 2 stream                       */
+  int64_t last_kernel;        /* 1 reference, 2 stream, 3 sequential         */
   int64_t last_grid;          /* CTAs of the last main launch                */
 } magus_stats;
 /* Synchronises when timing is on (reads the events). */

@@ -15,7 +15,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 BUILD = os.path.join(HERE, "build")
 LIB = os.path.join(HERE, "libmagus.so")
-SOURCES = ["api.cu", "precompute.cpp", "kernels_ref.cu", "kernels_stream.cu", "kernels_post.cu",
+SOURCES = ["api.cu", "precompute.cpp", "kernels_ref.cu", "kernels_seq.cu", "kernels_stream.cu", "kernels_post.cu",
            "kernels_bound.cu"]
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -32,7 +32,8 @@ def _nvcc() -> str:
 
 def _compile(src: str) -> tuple[str, str]:
     obj = os.path.join(BUILD, os.path.splitext(src)[0] + ".o")
-    cmd = [_nvcc(), *ARCH, *COMMON, "-x", "cu", "-c", os.path.join(CSRC, src), "-o", obj]
+    extra = os.environ.get("MAGUS_NVCC_FLAGS", "").split()  # developer experiments only
+    cmd = [_nvcc(), *ARCH, *COMMON, *extra, "-x", "cu", "-c", os.path.join(CSRC, src), "-o", obj]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"nvcc failed for {src}:\n{r.stdout}\n{r.stderr}")

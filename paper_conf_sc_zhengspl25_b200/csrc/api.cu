@@ -482,7 +482,7 @@ magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value) {
   if (!ctx) return MAGUS_ERR_INVALID_ARG;
   switch (key) {
     case MAGUS_OPT_KERNEL:
-      if (value < 0 || value > 2) return fail(ctx, MAGUS_ERR_INVALID_ARG, "kernel option %lld", (long long)value);
+      if (value < 0 || value > 3) return fail(ctx, MAGUS_ERR_INVALID_ARG, "kernel option %lld", (long long)value);
       ctx->opt_kernel = value;
       return MAGUS_OK;
     case MAGUS_OPT_SEGMENTS:
@@ -529,15 +529,22 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
   // kernel choice: the stream kernel runs the paper's MAGUS (variant 0) with
   // W <= 33, H <= 32 on TMA-addressable traces; everything else, and any
   // per-interval level output, runs the per-sample kernel
-  bool all_stream = out_levels == nullptr, multi = false;
+  bool all_stream = out_levels == nullptr, multi = false, closed = false, all_seq = true;
   for (int32_t c = 0; c < C; ++c) {
     all_stream = all_stream && params[c].variant == 0 &&
                  stream_supported(params[c].window, params[c].history);
     multi = multi || (params[c].variant & MAGUS_VARIANT_GRADUAL) != 0;
+    closed = closed || (params[c].variant & MAGUS_VARIANT_CLOSED_LOOP) != 0;
+    all_seq = all_seq && seq_supported(params[c]);
   }
   const bool tma_ok = ((uintptr_t)traces % 16 == 0) && (ld % 4 == 0);
+  all_seq = all_seq && ld < (int64_t(1) << 26);  // the sequential kernel's 32-bit row offsets
   int kernel = (int)ctx->opt_kernel;
-  if (kernel == 0) kernel = (all_stream && tma_ok) ? 2 : 1;
+  if (kernel == 0) kernel = (all_stream && tma_ok) ? 2 : (all_seq ? 3 : 1);
+  if (kernel == 3 && !all_seq)
+    return fail(ctx, MAGUS_ERR_UNSUPPORTED,
+                "sequential kernel: closed-loop configs need W <= 64 (jump) or W <= 128 (gradual), "
+                "and ld < 2^26");
   if (kernel == 2 && !(all_stream && tma_ok))
     return fail(ctx, MAGUS_ERR_UNSUPPORTED,
                 "stream kernel needs W in [2,33], H in [1,32], 16-B aligned traces and ld %% 4 == 0");
@@ -608,8 +615,8 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     ev1 = take_event(ctx);
   }
   int launched = 0;
-  if (kernel == 1) {
-    // the reference kernel writes summaries directly; totals need them
+  if (kernel == 1 || kernel == 3) {
+    // the per-sample kernels write summaries directly; totals need them
     const size_t sum_bytes = (out_summary || !out_totals) ? 0 : align_up(sizeof(magus_summary) * (size_t)(N * C), 256);
     const size_t base_bytes = (out_base || !out_totals) ? 0 : align_up(sizeof(magus_base) * (size_t)N, 256);
     st = ensure_scratch(ctx, sum_bytes + base_bytes + 256);
@@ -621,14 +628,22 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     magus_base* base = out_base;
     if (!base && out_totals) base = (magus_base*)sp;
     if (ctx->opt_timing) CK(cudaEventRecord(ev0, ctx->stream));
-    int r = launch_reference(ctx->stream, traces, N, T, ld, dev_policies(ctx), C, ctx->dplat,
-                             ctx->plat.bw_max_mbs, ctx->plat.p_other_w + ctx->plat.p_unc_min_w,
-                             ctx->plat.p_unc_max_w - ctx->plat.p_unc_min_w, multi,
-                             /*literal=*/ctx->opt_kernel == 1, summ, base,
-                             out_decisions, out_levels);
-    if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "reference kernel launch");
+    const double p_lo = ctx->plat.p_other_w + ctx->plat.p_unc_min_w;
+    const double p_span = ctx->plat.p_unc_max_w - ctx->plat.p_unc_min_w;
+    int r;
+    if (kernel == 3) {
+      r = launch_seq(ctx->stream, traces, N, T, ld, dev_policies(ctx), C, ctx->dplat,
+                     ctx->plat.bw_max_mbs, p_lo, p_span, closed, multi, summ, base, out_decisions,
+                     out_levels);
+      ctx->last_grid = (N * C + 31) / 32;
+    } else {
+      r = launch_reference(ctx->stream, traces, N, T, ld, dev_policies(ctx), C, ctx->dplat,
+                           ctx->plat.bw_max_mbs, p_lo, p_span, multi,
+                           /*literal=*/ctx->opt_kernel == 1, summ, base, out_decisions, out_levels);
+      ctx->last_grid = (N * C + 127) / 128;
+    }
+    if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "per-sample kernel launch");
     launched += r;
-    ctx->last_grid = (N * C + 127) / 128;
     if (ctx->opt_timing) CK(cudaEventRecord(ev1, ctx->stream));
     if (out_totals) {
       r = launch_totals(ctx->stream, summ, base, N, T, C, out_totals);

@@ -103,6 +103,14 @@ int launch_reference(cudaStream_t s, const float* x, int64_t N, int64_t T, int64
                      double p_lo, double p_span, bool multi, bool literal, magus_summary* out_summary,
                      magus_base* out_base, uint32_t* out_dec, uint8_t* out_levels);
 
+// Sequential-variant kernel (kernels_seq.cu): one thread per (trace, config),
+// cp.async-prefetched, latency-optimised chain; f3/f4 and level output.
+bool seq_supported(const magus_policy& p);
+int launch_seq(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,
+               const DevPolicy* pol_dev, int32_t C, const DevPlatform& plat, double bw_max,
+               double p_lo, double p_span, bool closed, bool multi, magus_summary* out_summary,
+               magus_base* out_base, uint32_t* out_dec, uint8_t* out_levels);
+
 bool stream_supported(int32_t W, int32_t H);
 // Fused stream kernel over nbund bundles of NB configs (bundles_dev:
 // [nbund][NB] global config indices, -1 = padding).  All configs of a launch
