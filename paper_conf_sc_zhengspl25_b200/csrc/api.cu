@@ -538,13 +538,14 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     all_seq = all_seq && seq_supported(params[c]);
   }
   const bool tma_ok = ((uintptr_t)traces % 16 == 0) && (ld % 4 == 0);
-  all_seq = all_seq && ld < (int64_t(1) << 26);  // the sequential kernel's 32-bit row offsets
+  all_seq = all_seq && ld < (int64_t(1) << 26)  // the sequential kernel's 32-bit row offsets
+            && seq_fits(ctx->dplat, closed, multi);  // per-ratio rows of wide ratio ranges
   int kernel = (int)ctx->opt_kernel;
   if (kernel == 0) kernel = (all_stream && tma_ok) ? 2 : (all_seq ? 3 : 1);
   if (kernel == 3 && !all_seq)
     return fail(ctx, MAGUS_ERR_UNSUPPORTED,
                 "sequential kernel: closed-loop configs need W <= 64 (jump) or W <= 128 (gradual), "
-                "and ld < 2^26");
+                "ld < 2^26, and a ratio range whose per-ratio rows fit in shared memory");
   if (kernel == 2 && !(all_stream && tma_ok))
     return fail(ctx, MAGUS_ERR_UNSUPPORTED,
                 "stream kernel needs W in [2,33], H in [1,32], 16-B aligned traces and ld %% 4 == 0");

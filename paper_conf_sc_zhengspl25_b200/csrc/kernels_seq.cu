@@ -13,7 +13,7 @@
 // With ~4k recurrences on 148 SMs the time is the latency of ONE chain per
 // step, so the kernel takes everything that does not depend on the
 // decisions off that chain (warp specialisation, one CTA per 32 traces):
-//   * 6 producer warps, round-robin over 32-step words: the samples x[t] and
+//   * 9 producer warps, round-robin over 32-step words: the samples x[t] and
 //     the Alg. 1 lags x[t-W+1] of the word (64 independent loads per lane),
 //     then the decision-independent predicates: the Alg. 1 outcomes as masks
 //     -- for the binary closed loop all four outcomes (interval t at r_min /
@@ -48,11 +48,12 @@ namespace {
 
 constexpr int kLanes = 32;         // traces per CTA (one lane each)
 constexpr int kWord = 32;          // steps per slot (= one decision word)
-constexpr int kProducers = 6;
+constexpr int kProducers = 9;
 constexpr int kAccountants = 3;
-// 12 warps: 0 consumer (alone on SMSP 0: 4 and 8 idle), 1/5/9 accountants
-// (SMSP 1), 2/3/6/7/10/11 producers (SMSPs 2 and 3)
-constexpr int kThreads = 32 * 12;
+// 16 warps, by SMSP (warp % 4): SMSP 0 = the consumer (warp 0) alone (4, 8,
+// 12 idle); SMSP 1 = accountants 1, 5, 9 + producer 13; SMSPs 2 and 3 =
+// producers 2, 3, 6, 7, 10, 11, 14, 15
+constexpr int kThreads = 32 * 16;
 constexpr int kAccFieldsSeq = 12;  // partial sums combined at the end (see the accountant)
 constexpr int kRingL = 128;        // CLOSED && MULTI: ratios of the last 128 intervals
 constexpr int kMaxLv = 128;
@@ -60,8 +61,8 @@ constexpr int kMaxLv = 128;
 // slot layout (bytes)
 constexpr int kOffX = 0;                              // float [32 steps][32 lanes] samples
 constexpr int kOffCode = kOffX + 4 * kWord * kLanes;  // u32 [8][32] closed-binary outcome codes
-constexpr int kOffPM = kOffCode + 4 * 8 * kLanes;     // u32 [4][32] big, burst, inc, dec
-constexpr int kOffCM = kOffPM + 4 * 4 * kLanes;       // u32 [5][32] dec, leff|change, event, hi masks, dec[t0-1]
+constexpr int kOffPM = kOffCode + 4 * 8 * kLanes;     // u32 [5][32] big, burst, inc, dec, big-at-max
+constexpr int kOffCM = kOffPM + 4 * 5 * kLanes;       // u32 [5][32] dec, leff|change, event, hi masks, dec[t0-1]
 constexpr int kOffLv = kOffCM + 4 * 5 * kLanes;       // u8 [32][32] MULTI ratios dec[t0+i]
 constexpr int kOffL = kOffLv + kWord * kLanes;        // float [32][32] Alg. 1 lags (CLOSED && MULTI)
 template <bool CLOSED, bool MULTI>
@@ -182,9 +183,9 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
   };
 
   if (warp >= 4 && (warp & 3) == 0) return;   // keeps SMSP 0 for the consumer
-  if ((warp & 3) >= 2) {
+  if ((warp & 3) >= 2 || warp == 13) {
     // =========================== producers ===============================
-    const int p = (warp >> 2) * 2 + (warp & 1);   // warps 2,3,6,7,10,11 -> 0..5
+    const int p = warp == 13 ? 8 : (warp >> 2) * 2 + (warp & 1);   // warps 2,3,6,7,10,11,14,15,13 -> 0..8
     const float* xcol = a.x + n;
     // the closed loop is per config; an open-loop config observes through an
     // infinite capacity (delivered(x, inf) = x, NaN included)
@@ -192,7 +193,7 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
     const double obs_max = closed ? plat.Bmax : (double)INFINITY;
     const bool bursts = plat.burst_mbs > 0.0;
     const float xthr = plat.xthr_min;  // x <= xthr: no stretch at any ratio (B_l >= B_min)
-    // Each producer owns every 6th word.  Waiting on empty(j) needs word
+    // Each producer owns every 9th word.  Waiting on empty(j) needs word
     // j - kSlots < j to be accounted, which by induction on the word index
     // never waits on an unpublished word.
     const double d_inc = P.d_inc, d_dec = P.d_dec;
@@ -215,91 +216,96 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
         dn = D < d_dec;
       }
     };
+    const float xthrM = plat.xthr_max;  // x <= xthrM: no stretch at r_max
+    // Half-word pipeline: the 32 loads of the next half (this word's second
+    // half, or the first half of this producer's next word) are in flight
+    // while the current half is evaluated.
+    auto load_half = [&](int64_t jj, int h, float (&xv)[16], float (&lg)[16]) {
+      if (jj >= nwords) return;
+      const int64_t t0 = jj * kWord + 16 * h;
+      const int cnt = word_cnt(jj);
+      const uint32_t live = cnt == 32 ? 0xFFFFFFFFu : ((1u << cnt) - 1u);
+      const uint32_t mdfs = word_mdfs(jj, live) >> (16 * h), lv = live >> (16 * h);
+      const float* src = xcol + t0 * a.ld;
+      const float* lsrc = xcol + (t0 - W + 1) * a.ld;
+      if (__all_sync(0xFFFFFFFFu, (mdfs & 0xFFFFu) == 0xFFFFu)) {
+#pragma unroll
+        for (int u = 0; u < 16; ++u) {
+          xv[u] = __ldg(src + u * ld32);
+          lg[u] = __ldg(lsrc + u * ld32);
+        }
+      } else {
+#pragma unroll
+        for (int u = 0; u < 16; ++u) {
+          xv[u] = ((lv >> u) & 1) ? __ldg(src + u * ld32) : 0.0f;
+          lg[u] = ((mdfs >> u) & 1) ? __ldg(lsrc + u * ld32) : 0.0f;
+        }
+      }
+    };
+    float cx[16], cl[16];
+    load_half(p, 0, cx, cl);
     for (int64_t j = p; j < nwords; j += kProducers) {
       const int s = (int)(j % kSlots);
       unsigned char* sl = slots + s * kSlotBytes;
-      const int64_t t0 = j * kWord;
       const int cnt = word_cnt(j);
       const uint32_t live = cnt == 32 ? 0xFFFFFFFFu : ((1u << cnt) - 1u);
       const uint32_t mdfs = word_mdfs(j, live);
-      uint32_t big = 0, brst = 0, inc = 0, dcr = 0;
-      const float* src = xcol + t0 * a.ld;
-      const float* lsrc = xcol + (t0 - W + 1) * a.ld;
+      uint32_t big = 0, bigM = 0, brst = 0, inc = 0, dcr = 0;
       float* xs = reinterpret_cast<float*>(sl + kOffX) + lane;
       uint32_t* cwp = reinterpret_cast<uint32_t*>(sl + kOffCode) + lane;
-      if (__all_sync(0xFFFFFFFFu, cnt == kWord && t0 >= W) && !(CLOSED && MULTI)) {
-        // whole word, all MDFS rounds: 64 loads in flight, then the slot
-        float xv[kWord], lg[kWord];
-#pragma unroll
-        for (int i = 0; i < kWord; ++i) {
-          xv[i] = __ldg(src + i * ld32);
-          lg[i] = __ldg(lsrc + i * ld32);
-        }
-        if (j >= kSlots) reclaim(j);
-#pragma unroll
-        for (int i = 0; i < kWord; ++i) xs[i * kLanes] = xv[i];
-        uint32_t cw = 0;
-#pragma unroll
-        for (int i = 0; i < (SEQ_ABLATE == 2 ? 0 : kWord); ++i) {
-          big |= (uint32_t)(xv[i] > xthr) << i;
-          brst |= (uint32_t)(xv[i] > xburst) << i;
-          uint32_t cd = 0, up = 0, dn = 0;
-          eval(xv[i], lg[i], cd, up, dn);
-          if constexpr (CLOSED) {
-            cw |= cd << (8 * (i & 3));
-            if ((i & 3) == 3) {
-              cwp[(i >> 2) * kLanes] = cw;
-              cw = 0;
-            }
-          } else {
-            inc |= up << i;
-            dcr |= dn << i;
-          }
-        }
-      } else {
-        if (j >= kSlots) reclaim(j);
 #pragma unroll 1
-        for (int h = 0; h < kWord; h += 16) {   // two halves of 16 steps: 32 loads in flight
-          float xv[16], lg[16];
+      for (int h = 0; h < 2; ++h) {
+        float nx[16], nl[16];
+        if (h == 0) load_half(j, 1, nx, nl);
+        else load_half(j + kProducers, 0, nx, nl);
+        if (h == 0 && j >= kSlots) reclaim(j);
 #pragma unroll
-          for (int u = 0; u < 16; ++u) {
-            const int i = h + u;
-            xv[u] = ((live >> i) & 1) ? __ldg(src + i * ld32) : 0.0f;
-            lg[u] = ((mdfs >> i) & 1) ? __ldg(lsrc + i * ld32) : 0.0f;
+        for (int u = 0; u < 16; ++u) xs[(16 * h + u) * kLanes] = cx[u];
+        if constexpr (CLOSED && MULTI) {
+          float* ls = reinterpret_cast<float*>(sl + kOffL) + lane;
+#pragma unroll
+          for (int u = 0; u < 16; ++u) ls[(16 * h + u) * kLanes] = cl[u];
+        }
+        const uint32_t rd16 = (mdfs >> (16 * h)) & 0xFFFFu;
+        uint32_t b16 = 0, bm16 = 0, r16 = 0, i16 = 0, d16 = 0, cw = 0;
+#pragma unroll
+        for (int u = 0; u < 16; ++u) {
+          const float xt = cx[u];
+          b16 |= (uint32_t)(xt > xthr) << u;
+          bm16 |= (uint32_t)(xt > xthrM) << u;
+          r16 |= (uint32_t)(xt > xburst) << u;
+          if (!(CLOSED && MULTI) && ((rd16 >> u) & 1)) {
+            uint32_t cd = 0, up = 0, dn = 0;
+            eval(xt, cl[u], cd, up, dn);
+            cw |= cd << (8 * (u & 3));
+            i16 |= up << u;
+            d16 |= dn << u;
           }
-#pragma unroll
-          for (int u = 0; u < 16; ++u) xs[(h + u) * kLanes] = xv[u];
-          if constexpr (CLOSED && MULTI) {
-            float* ls = reinterpret_cast<float*>(sl + kOffL) + lane;
-#pragma unroll
-            for (int u = 0; u < 16; ++u) ls[(h + u) * kLanes] = lg[u];
+          if (CLOSED && !MULTI && (u & 3) == 3) {
+            cwp[(4 * h + (u >> 2)) * kLanes] = cw;
+            cw = 0;
           }
-          uint32_t cw = 0;
+        }
+        big |= b16 << (16 * h);
+        bigM |= bm16 << (16 * h);
+        brst |= r16 << (16 * h);
+        inc |= i16 << (16 * h);
+        dcr |= d16 << (16 * h);
 #pragma unroll
-          for (int u = 0; u < 16; ++u) {
-            const int i = h + u;
-            const float xt = xv[u];
-            big |= (uint32_t)(xt > xthr) << i;
-            brst |= (uint32_t)(xt > xburst) << i;
-            if (!(CLOSED && MULTI) && ((mdfs >> i) & 1)) {
-              uint32_t cd = 0, up = 0, dn = 0;
-              eval(xt, lg[u], cd, up, dn);
-              cw |= cd << (8 * (u & 3));
-              inc |= up << i;
-              dcr |= dn << i;
-            }
-            if (CLOSED && !MULTI && (u & 3) == 3) {
-              cwp[((h + u) >> 2) * kLanes] = cw;
-              cw = 0;
-            }
-          }
+        for (int u = 0; u < 16; ++u) {
+          cx[u] = nx[u];
+          cl[u] = nl[u];
         }
       }
+      big &= live;
+      bigM &= live;
+      brst &= live;
       uint32_t* pm = reinterpret_cast<uint32_t*>(sl + kOffPM) + lane;
       pm[0] = big;
       pm[kLanes] = brst;
       pm[2 * kLanes] = inc;
       pm[3 * kLanes] = dcr;
+      pm[4 * kLanes] = bigM;
       warp_arrive(full(s));
     }
     return;
@@ -489,20 +495,23 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
   }
 
   // ============================= accountants ============================
-  // kAccountants warps take the words round-robin; every quantity is a sum
-  // over words (per-level model-M rows are shared and updated with shared-
-  // memory atomics), combined by accountant 0 at the end.
+  // kAccountants warps take the words round-robin; every quantity is an
+  // integer sum over words (per-level model-M rows private to each
+  // accountant), combined by accountant 0 at the end.
   const int acc_id = warp >> 2;      // warps 1, 5, 9 -> 0, 1, 2
   const bool bursts = plat.burst_mbs > 0.0;
   const int burst_at_max = plat.Bmax > plat.burst_mbs, burst_at_min = plat.Bmin > plat.burst_mbs;
   const double invB_min = plat.invB_min, invB_max = plat.invB_max;
   unsigned char* tail = slots + kSlots * kSlotBytes + (CLOSED && MULTI ? kRingL * kLanes : 0);
-  unsigned long long* qacc = reinterpret_cast<unsigned long long*>(tail);               // MULTI [nlev][32]
-  uint32_t* nacc = reinterpret_cast<uint32_t*>(qacc + (MULTI ? nlev * kLanes : 0));      // MULTI [nlev][32]
-  unsigned long long* part = reinterpret_cast<unsigned long long*>(nacc + (MULTI ? nlev * kLanes : 0));
+  // MULTI: qacc [kAccountants][nlev][32] u64, nacc [kAccountants][nlev][32] u32
+  unsigned long long* qacc0 = reinterpret_cast<unsigned long long*>(tail);
+  uint32_t* nacc0 = reinterpret_cast<uint32_t*>(qacc0 + (MULTI ? kAccountants * nlev * kLanes : 0));
+  unsigned long long* part = reinterpret_cast<unsigned long long*>(nacc0 + (MULTI ? kAccountants * nlev * kLanes : 0));
   // part: [kAccountants - 1][kAccFieldsSeq][32] partial sums of accountants 1..
+  unsigned long long* qacc = qacc0 + (size_t)acc_id * nlev * kLanes;
+  uint32_t* nacc = nacc0 + (size_t)acc_id * nlev * kLanes;
   if constexpr (MULTI) {
-    for (int i = acc_id; i < nlev; i += kAccountants) {
+    for (int i = 0; i < nlev; ++i) {
       qacc[i * kLanes + lane] = 0;
       nacc[i * kLanes + lane] = 0;
     }
@@ -527,7 +536,7 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
     const uint32_t* pm = reinterpret_cast<const uint32_t*>(sl + kOffPM) + lane;
     const uint32_t* cm = reinterpret_cast<const uint32_t*>(sl + kOffCM) + lane;
     const float* xs = reinterpret_cast<const float*>(sl + kOffX) + lane;
-    const uint32_t big = pm[0] & live, brst = pm[kLanes] & live;
+    const uint32_t big = pm[0] & live, brst = pm[kLanes] & live, bigM = pm[4 * kLanes] & live;
     const uint32_t decm = cm[0] & live, m1 = cm[kLanes] & live, evm = cm[2 * kLanes], him = cm[3 * kLanes];
     events += __popc(evm);
     hi_rounds += __popc(him);
@@ -547,14 +556,14 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
       if (active) {
         uint32_t cb = m1;
         int pos = 0, g = lin;
-        while (cb) {                   // runs of g (ratio changes are rare)
+        while (cb) {                   // runs of g (one per ratio change)
           const int i = __ffs(cb) - 1;
           cb &= cb - 1;
-          atomicAdd(&nacc[(g - lmin) * kLanes + lane], (uint32_t)(i + 1 - pos));
+          nacc[(g - lmin) * kLanes + lane] += (uint32_t)(i + 1 - pos);
           g = lvw[i * kLanes];
           pos = i + 1;
         }
-        if (cnt > pos) atomicAdd(&nacc[(g - lmin) * kLanes + lane], (uint32_t)(cnt - pos));
+        if (cnt > pos) nacc[(g - lmin) * kLanes + lane] += (uint32_t)(cnt - pos);
         uint32_t bm = big | brst;
         while (bm) {                   // samples above the capacity at r_min / bursts (sparse)
           const int i = __ffs(bm) - 1;
@@ -562,10 +571,10 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
           const int gi = i == 0 ? lin : (int)lvw[(i - 1) * kLanes];
           const float xt = xs[i * kLanes];
           if ((big >> i) & 1) {
-            const uint64_t qb = q_at(xt, invB_max);
+            const uint64_t qb = ((bigM >> i) & 1) ? q_scaled(xt, invB_max * kQScale) : 0ull;
             q_base += qb;
             const uint64_t q = gi == lmax ? qb : q_at(xt, s_invB[gi - lmin]);
-            if (q) atomicAdd(&qacc[(gi - lmin) * kLanes + lane], (unsigned long long)q);
+            qacc[(gi - lmin) * kLanes + lane] += q;
           }
           if ((brst >> i) & 1) {       // delivered min(x, B_l) > theta
             b_base += burst_at_max;
@@ -591,9 +600,9 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
         const int i = __ffs(bm) - 1;
         bm &= bm - 1;
         const float xt = xs[i * kLanes];
-        const uint64_t qb = q_at(xt, invB_max);
+        const uint64_t qb = ((bigM >> i) & 1) ? q_scaled(xt, invB_max * kQScale) : 0ull;
         q_base += qb;
-        if ((m1 >> i) & 1) q_min += q_at(xt, invB_min);
+        if ((m1 >> i) & 1) q_min += q_scaled(xt, invB_min * kQScale);   // big: x > xthr_min
         else q_max += qb;
       }
       if (bursts) {
@@ -632,10 +641,15 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
   }
   magus_summary* so = a.summary ? a.summary + (int64_t)c * a.N + n : nullptr;
   magus_base* bo = (a.base && c == 0) ? a.base + n : nullptr;
-  if constexpr (MULTI) {
-    n_min_int = (int32_t)nacc[lane];
-    q_min = qacc[lane];
-    for (int i = 1; i < nlev; ++i) q_max += qacc[i * kLanes + lane];
+  if constexpr (MULTI) {   // per-level rows: sum over the accountants (integers)
+    for (int w = 1; w < kAccountants; ++w)
+      for (int i = 0; i < nlev; ++i) {
+        qacc0[i * kLanes + lane] += qacc0[((size_t)w * nlev + i) * kLanes + lane];
+        nacc0[i * kLanes + lane] += nacc0[((size_t)w * nlev + i) * kLanes + lane];
+      }
+    n_min_int = (int32_t)nacc0[lane];
+    q_min = qacc0[lane];
+    for (int i = 1; i < nlev; ++i) q_max += qacc0[i * kLanes + lane];
   }
   finalize_summary(plat, T, events, hi_rounds, msr, changes, n_min_dec, n_min_int, q_min, q_max, q_base,
                    digest, b_base, b_magus, so, bo);
@@ -645,8 +659,8 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
       for (int i = 0; i < nlev; ++i) {
         const int l = lmin + i;
         const double Pl = a.p_lo + (a.p_span * (double)(l - lmin)) / (double)(lmax - lmin);
-        energy = energy + Pl * (plat.dt * (double)nacc[i * kLanes + lane] +
-                                plat.cQ * (double)qacc[i * kLanes + lane]);
+        energy = energy + Pl * (plat.dt * (double)nacc0[i * kLanes + lane] +
+                                plat.cQ * (double)qacc0[i * kLanes + lane]);
       }
       so->energy_j = energy + plat.e_sw * (double)changes;
     }
@@ -659,12 +673,19 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
 #undef tok
 
 template <bool CLOSED, bool MULTI>
-int launch_one(cudaStream_t s, const SeqArgs& a, const DevPlatform& plat) {
+size_t smem_bytes(const DevPlatform& plat) {
   const int nlev = plat.r_max - plat.r_min + 1;
   size_t smem = (size_t)n_slots<CLOSED, MULTI>() * slot_bytes<CLOSED, MULTI>();
   if (CLOSED && MULTI) smem += (size_t)kRingL * kLanes;
-  if (MULTI) smem += (size_t)nlev * kLanes * (sizeof(uint64_t) + sizeof(uint32_t));
+  if (MULTI) smem += (size_t)kAccountants * nlev * kLanes * (sizeof(uint64_t) + sizeof(uint32_t));
   smem += (size_t)(kAccountants - 1) * kAccFieldsSeq * kLanes * sizeof(uint64_t);
+  return smem;
+}
+constexpr size_t kSmemLimit = 227 * 1024;
+
+template <bool CLOSED, bool MULTI>
+int launch_one(cudaStream_t s, const SeqArgs& a, const DevPlatform& plat) {
+  const size_t smem = smem_bytes<CLOSED, MULTI>(plat);
   auto k = seq_kernel<CLOSED, MULTI>;
   if (smem > 48 * 1024 &&
       cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
@@ -676,6 +697,12 @@ int launch_one(cudaStream_t s, const SeqArgs& a, const DevPlatform& plat) {
 }
 
 }  // namespace
+
+bool seq_fits(const DevPlatform& plat, bool closed, bool multi) {
+  const size_t b = closed ? (multi ? smem_bytes<true, true>(plat) : smem_bytes<true, false>(plat))
+                          : (multi ? smem_bytes<false, true>(plat) : smem_bytes<false, false>(plat));
+  return b <= kSmemLimit;
+}
 
 bool seq_supported(const magus_policy& p) {
   if (!(p.variant & MAGUS_VARIANT_CLOSED_LOOP)) return true;

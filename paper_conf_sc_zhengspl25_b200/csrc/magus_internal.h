@@ -106,6 +106,7 @@ int launch_reference(cudaStream_t s, const float* x, int64_t N, int64_t T, int64
 // Sequential-variant kernel (kernels_seq.cu): one thread per (trace, config),
 // cp.async-prefetched, latency-optimised chain; f3/f4 and level output.
 bool seq_supported(const magus_policy& p);
+bool seq_fits(const DevPlatform& plat, bool closed, bool multi);  // shared memory of the launch
 int launch_seq(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,
                const DevPolicy* pol_dev, int32_t C, const DevPlatform& plat, double bw_max,
                double p_lo, double p_span, bool closed, bool multi, magus_summary* out_summary,
