@@ -321,7 +321,10 @@ def run_ours(args):
     alg_bytes = N * T * 4 + (C * N * T / 8 if want_dec else 0)
     achieved = alg_bytes / (kern_ms * 1e-3) / 1e9
     traffic = None
-    prof = os.path.join(ROOT, "profiles", f"ncu_cfg{args.config}.json")
+    kname = {1: "ref_kernel", 2: "stream_kernel", 3: "seq_kernel"}.get(st["last_kernel"], "?")
+    vtag = {0: "", 1: "_f3", 2: "_f4"}.get(args.variant, f"_v{args.variant}")
+    # traffic only from an ncu capture of this very kernel and workload
+    prof = os.path.join(ROOT, "profiles", f"ncu_cfg{args.config}{vtag}.json")
     if os.path.exists(prof):
         try:
             with open(prof) as f:
@@ -380,7 +383,7 @@ def run_ours(args):
     clk = clocks.summary()
     hbm_roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                "kernel": "stream_kernel", "kernel_ms": kern_ms, "alg_bytes_per_launch": alg_bytes}
+                "kernel": kname, "kernel_ms": kern_ms, "alg_bytes_per_launch": alg_bytes}
     roof = hbm_roof
     if C > 1:
         sm_mhz = clk.get("sm_max_mhz") or 1965.0
@@ -389,7 +392,7 @@ def run_ours(args):
         roof = {"bound": "alu", "achieved": alu_ach, "peak": alu_peak, "unit": "Gop/s",
                 "frac": alu_ach / alu_peak, "traffic": traffic,
                 "peak_source": f"148 SMs x 128 lanes x {sm_mhz:.0f} MHz (B200_PROFILING.md unit counts)",
-                "kernel": "stream_kernel", "kernel_ms": kern_ms, "alg_ops_per_decision": 8}
+                "kernel": kname, "kernel_ms": kern_ms, "alg_ops_per_decision": 8}
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
