@@ -321,7 +321,7 @@ def run_ours(args):
     alg_bytes = N * T * 4 + (C * N * T / 8 if want_dec else 0)
     achieved = alg_bytes / (kern_ms * 1e-3) / 1e9
     traffic = None
-    kname = {1: "ref_kernel", 2: "stream_kernel", 3: "seq_kernel"}.get(st["last_kernel"], "?")
+    kname = {1: "ref_kernel", 2: "stream_kernel", 3: "seq_kernel", 4: "walk_replay_kernel"}.get(st["last_kernel"], "?")
     vtag = {0: "", 1: "_f3", 2: "_f4"}.get(args.variant, f"_v{args.variant}")
     # traffic only from an ncu capture of this very kernel and workload
     prof = os.path.join(ROOT, "profiles", f"ncu_cfg{args.config}{vtag}.json")
@@ -400,7 +400,7 @@ def run_ours(args):
                        "n_configs": C, "decisions_emitted": want_dec, "seed": hex(seed),
                        "l2": f"inputs {N * T * 4 / 1e9:.2f} GB per GPU > 126 MB L2 (no flush needed)",
                        "parallelism": f"traces sharded over {world} GPU(s); 1 all-reduce of int64 totals ({dist_backend(world)})",
-                       "segments": st["last_segments"], "kernel": {1: "reference", 2: "stream", 3: "sequential"}.get(st["last_kernel"], "?"),
+                       "segments": st["last_segments"], "kernel": {1: "reference", 2: "stream", 3: "sequential", 4: "walk"}.get(st["last_kernel"], "?"),
                        "variant": args.variant, "step": args.step if args.variant & 2 else 0},
             "roofline": roof,
             "cpu_baseline": cpu, "e2e": e2e,

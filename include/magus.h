@@ -390,9 +390,10 @@ magus_status magus_platform_inspect(const magus_platform* p, magus_platform_cons
 enum {
   MAGUS_OPT_KERNEL = 0,       /* 0 auto, 1 reference (per-sample, the printed
                                  divisions), 2 stream, 3 sequential (per-sample,
-                                 latency-optimised: f3/f4 and level output;
-                                 the auto choice when the stream kernel cannot
-                                 run)                                        */
+                                 latency-optimised: the auto choice for the
+                                 closed loop f3), 4 walk (time-segmented
+                                 open loop: the auto choice for f4 and level
+                                 output; UNSUPPORTED for closed-loop configs) */
   MAGUS_OPT_SEGMENTS = 1,     /* 0 auto, else the number of time segments    */
   MAGUS_OPT_TIMING = 2,       /* 1: record CUDA events around the main kernel */
   MAGUS_OPT_WAVES = 3,        /* auto segmentation: 0 (default) = wave model

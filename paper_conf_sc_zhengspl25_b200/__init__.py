@@ -25,7 +25,7 @@ POLICY_PAPER_DEFAULT, POLICY_PAPER_PARETO = 0, 1
 PLATFORM_INTEL_A100, PLATFORM_INTEL_MAX1550 = 0, 1
 GEN_MIX, GEN_ADVERSARIAL = 0, 1
 OPT_KERNEL, OPT_SEGMENTS, OPT_TIMING, OPT_WAVES, OPT_BUNDLE = 0, 1, 2, 3, 4
-KERNEL_AUTO, KERNEL_REFERENCE, KERNEL_STREAM, KERNEL_SEQUENTIAL = 0, 1, 2, 3
+KERNEL_AUTO, KERNEL_REFERENCE, KERNEL_STREAM, KERNEL_SEQUENTIAL, KERNEL_WALK = 0, 1, 2, 3, 4
 TOT_WORDS = 18
 TOT_NAMES = ["n_traces", "n_viol", "events", "hi_rounds", "msr_writes", "changes", "min_dec",
              "min_int", "qmin_lo", "qmin_hi", "qmax_lo", "qmax_hi", "qbase_lo", "qbase_hi",

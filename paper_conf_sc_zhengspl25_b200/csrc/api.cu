@@ -482,7 +482,7 @@ magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value) {
   if (!ctx) return MAGUS_ERR_INVALID_ARG;
   switch (key) {
     case MAGUS_OPT_KERNEL:
-      if (value < 0 || value > 3) return fail(ctx, MAGUS_ERR_INVALID_ARG, "kernel option %lld", (long long)value);
+      if (value < 0 || value > 4) return fail(ctx, MAGUS_ERR_INVALID_ARG, "kernel option %lld", (long long)value);
       ctx->opt_kernel = value;
       return MAGUS_OK;
     case MAGUS_OPT_SEGMENTS:
@@ -541,7 +541,12 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
   all_seq = all_seq && ld < (int64_t(1) << 26)  // the sequential kernel's 32-bit row offsets
             && seq_fits(ctx->dplat, closed, multi);  // per-ratio rows of wide ratio ranges
   int kernel = (int)ctx->opt_kernel;
-  if (kernel == 0) kernel = (all_stream && tma_ok) ? 2 : (all_seq ? 3 : 1);
+  // open loop (no closed-loop config): the time-segmented walk kernel
+  const bool walk_ok = !closed && ld < (int64_t(1) << 26);  // 32-bit row offsets of a 32-step word
+  if (kernel == 0) kernel = (all_stream && tma_ok) ? 2 : (walk_ok ? 4 : (all_seq ? 3 : 1));
+  if (kernel == 4 && !walk_ok)
+    return fail(ctx, MAGUS_ERR_UNSUPPORTED,
+                "walk kernel: closed-loop configs (variant 1, 3) have no exact time segmentation; ld < 2^26");
   if (kernel == 3 && !all_seq)
     return fail(ctx, MAGUS_ERR_UNSUPPORTED,
                 "sequential kernel: closed-loop configs need W <= 64 (jump) or W <= 128 (gradual), "
@@ -616,7 +621,48 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     ev1 = take_event(ctx);
   }
   int launched = 0;
-  if (kernel == 1 || kernel == 3) {
+  if (kernel == 4) {
+    // segments: enough independent (trace, segment, config) chains for about
+    // two full waves of resident threads, each >= 256 steps (halo re-read
+    // and map composition stay a few per cent)
+    if (ctx->opt_segments > 0) {
+      nseg = ctx->opt_segments;
+    } else {
+      const int64_t target = (int64_t)ctx->sms * 2048 * 2;
+      nseg = std::max<int64_t>(1, (target + N * C - 1) / (N * C));
+      nseg = std::min<int64_t>(nseg, std::max<int64_t>(1, T / 256));
+    }
+    nseg = std::min<int64_t>(std::max<int64_t>(nseg, 1), 65535);
+    seg_len = ((T + nseg - 1) / nseg + 31) / 32 * 32;
+    nseg = (T + seg_len - 1) / seg_len;
+    const size_t sum_bytes = out_summary ? 0 : align_up(sizeof(magus_summary) * (size_t)(N * C), 256);
+    const size_t base_bytes = (out_base || !out_totals) ? 0 : align_up(sizeof(magus_base) * (size_t)N, 256);
+    const size_t walk_bytes = walk_scratch_bytes(N, C, T, nseg, ctx->dplat);
+    int32_t max_H = 1;
+    for (int32_t c = 0; c < C; ++c) max_H = std::max(max_H, params[c].history);
+    st = ensure_scratch(ctx, sum_bytes + base_bytes + walk_bytes + 256);
+    if (st != MAGUS_OK) return st;
+    ctx->work_sig = 0;  // scratch reused: the stream path must re-zero its counters
+    char* sp = (char*)ctx->scratch;
+    magus_summary* summ = out_summary;
+    if (!summ) { summ = (magus_summary*)sp; sp += sum_bytes; }
+    magus_base* base = out_base;
+    if (!base && out_totals) { base = (magus_base*)sp; sp += base_bytes; }
+    if (ctx->opt_timing) CK(cudaEventRecord(ev0, ctx->stream));
+    const double p_lo = ctx->plat.p_other_w + ctx->plat.p_unc_min_w;
+    const double p_span = ctx->plat.p_unc_max_w - ctx->plat.p_unc_min_w;
+    int r = launch_walk(ctx->stream, traces, N, T, ld, dev_policies(ctx), C, max_H, ctx->dplat, ctx->plat.bw_max_mbs,
+                        p_lo, p_span, nseg, seg_len, sp, summ, base, out_decisions, out_levels);
+    if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "walk kernel launch");
+    launched += r;
+    ctx->last_grid = ((N + 127) / 128) * nseg * C;
+    if (ctx->opt_timing) CK(cudaEventRecord(ev1, ctx->stream));
+    if (out_totals) {
+      r = launch_totals(ctx->stream, summ, base, N, T, C, out_totals);
+      if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "totals kernel launch");
+      launched += r;
+    }
+  } else if (kernel == 1 || kernel == 3) {
     // the per-sample kernels write summaries directly; totals need them
     const size_t sum_bytes = (out_summary || !out_totals) ? 0 : align_up(sizeof(magus_summary) * (size_t)(N * C), 256);
     const size_t base_bytes = (out_base || !out_totals) ? 0 : align_up(sizeof(magus_base) * (size_t)N, 256);

@@ -1,0 +1,387 @@
+// kernels_walk.cu -- the time-segmented replay of the open-loop variants:
+// NEXT f4 (gradual +-step rule, P@35554) and the paper's jump rule whenever
+// per-interval levels are requested.
+//
+// Why it segments exactly.  In the open loop, Alg. 1's outcome p_t and
+// Alg. 2's hi_t are pure functions of the trace (closed form);
+// only the level walk is sequential, and every round applies to the level
+// one map of the form
+//     l -> min(max(l + d, a), b)          (r_min <= a <= b <= r_max)
+// -- hold (d = 0, a = r_min, b = r_max), step up (Alg. 3 l.18 with the f4
+// step: min(l + s, r_max)), step down (l.23-25: max(l - s, r_min)), the
+// override to max (l.10: a = b = r_max).  These clamp-shift maps are closed
+// under composition: applying up-step s to (d, a, b) gives
+// (d + s, min(a + s, r_max), min(b + s, r_max)), down-step symmetrically,
+// and on the domain [r_min, r_max] every d beyond +-(r_max - r_min) acts like
+// the bound, so d saturates there.  A segment's whole effect on the carry is
+// therefore one packed 32-bit map.
+//
+// Three launches (plus the totals kernel of kernels_post.cu):
+//   walk_map_kernel     one thread per (trace, segment, config): rebuild the
+//                       event history of the H rounds before the segment
+//                       (the halo), compose the segment's map; segment-0
+//                       threads also zero the (config, trace) accumulators;
+//   walk_replay_kernel  same threads: carry-in = the composition of the maps
+//                       of all earlier segments applied to r_max (interval 0
+//                       runs at max, P@23755), then the rounds of the
+//                       segment in the paper's order with model-M accounting
+//                       at the level that governs each interval (dec[t-1],
+//                       reading R6); integer segment sums go into the
+//                       accumulators with 64-bit atomics (exact, any order);
+//                       per-level (intervals, stretch) pairs are
+//                       run-length accumulated and flushed on level changes;
+//   walk_final_kernel   one thread per (trace, config): model M (the general
+//                       per-level form of DESIGN.md 4.3, the fp64 order of
+//                       kernels_ref.cu) into the summaries.
+// Compared with the latency-optimised seq_kernel (one chain per trace), the
+// segments give ~10^5 independent chains, so the walk is throughput-bound;
+// the price is reading the traces twice.
+#include <algorithm>
+
+#include "device_common.cuh"
+
+namespace magus {
+namespace {
+
+constexpr int kWalkThreads = 128;
+constexpr int kWalkChunk = 16;   // samples (and lags) loaded ahead of the chain
+constexpr int kWalkMaxLv = 128;  // ratios 1..127
+
+enum { WF_EV, WF_HI, WF_MSR, WF_CH, WF_MDEC, WF_QBASE, WF_DIG, WF_BB, WF_BM, kWalkFields };
+
+struct WalkArgs {
+  const float* x;
+  int64_t N, ld;
+  int32_t T, nw;                 // intervals (<= 2^24), 32-step words
+  const DevPolicy* pol;
+  int32_t C, c0;                 // all configs; first config of this launch (grid z = batch)
+  int32_t nseg, seg_len;         // seg_len % 32 == 0
+  uint32_t* map;                 // [batch][nseg][N] packed segment maps
+  uint32_t* mask;                // [batch][3][nw][N] Alg. 1 +1 / -1 and Alg. 2 hi bits per round
+  unsigned long long* acc;       // [C][kWalkFields][N]
+  unsigned int* lvn;             // [C][nlev][N] intervals per level
+  unsigned long long* lvq;       // [C][nlev][N] stretch q per level
+  magus_summary* summary;        // [C][N] (required)
+  magus_base* base;              // [N] or NULL
+  uint32_t* dec;                 // [C][nw][N] or NULL
+  uint8_t* levels;               // [C][T][N] or NULL
+  double p_lo, p_span;
+};
+
+// per-level constants, host-computed (the same formulas as kernels_ref.cu);
+// passed by value (1.7 KB of kernel parameters)
+struct WalkLevels {
+  double invB[kWalkMaxLv];       // 1 / B_l
+  float xthr[kWalkMaxLv];        // x > xthr[l] <=> RN(x * invB[l]) > 1
+  uint8_t bkeep[kWalkMaxLv];     // B_l > theta (a burst stays a burst at l)
+};
+
+__device__ __forceinline__ uint32_t map_pack(int d, int a, int b) {
+  return (uint32_t)(uint8_t)(int8_t)d | ((uint32_t)a << 8) | ((uint32_t)b << 16);
+}
+__device__ __forceinline__ int map_apply(uint32_t m, int l) {
+  const int d = (int)(int8_t)(m & 0xFFu), a = (int)((m >> 8) & 0xFFu), b = (int)((m >> 16) & 0xFFu);
+  return min(max(l + d, a), b);
+}
+
+// uncore_tune_ls at the start of round t0: the events of rounds
+// max(W, t0 - H) .. t0 - 1 (bit j = round t0 - 1 - j); Alg. 1 with the
+// host-inverted thresholds (delta > d_inc <=> RN(delta / L) > tau_inc; NaN:
+// neither, reading R9)
+__device__ __forceinline__ uint64_t history_at(const WalkArgs& a, const DevPolicy& P, int64_t n, int32_t t0) {
+  uint64_t hist = 0;
+  for (int32_t t = max(P.W, t0 - P.H); t < t0; ++t) {
+    const double D = (double)a.x[(int64_t)t * a.ld + n] - (double)a.x[(int64_t)(t - P.W + 1) * a.ld + n];
+    hist = (hist << 1) | (uint64_t)(D > P.d_inc || D < P.d_dec);
+  }
+  return hist;
+}
+
+// 16 samples x[t0 + i * ld32 rows] (32-bit row offsets: ld < 2^26, checked
+// by the dispatcher, keeps every address one IMAD from the base)
+__device__ __forceinline__ void load16(const float* __restrict__ p, int ld32, float (&v)[kWalkChunk]) {
+#pragma unroll
+  for (int i = 0; i < kWalkChunk; ++i) v[i] = __ldg(p + i * ld32);
+}
+
+// Pass 1: per (trace, segment, config) thread, the rounds of the segment in
+// the paper's order -- Alg. 2 on the H previous events (s >= k <=> RN(s/H)
+// >= t_hi), Alg. 1 (host-inverted thresholds), event logging -- recorded as
+// three bit masks per 32-step word, and composed into the segment's map.
+template <typename HT>
+__global__ void __launch_bounds__(kWalkThreads, 4) walk_map_kernel(WalkArgs a, int32_t lmin, int32_t lmax, int32_t nlev) {
+  const int64_t n = (int64_t)blockIdx.x * kWalkThreads + threadIdx.x;
+  const int32_t s = blockIdx.y, cl = blockIdx.z, c = a.c0 + cl;
+  if (n >= a.N) return;
+  if (s == 0) {  // fresh accumulators for this replay
+    for (int f = 0; f < kWalkFields; ++f) a.acc[((int64_t)c * kWalkFields + f) * a.N + n] = 0ull;
+    for (int i = 0; i < nlev; ++i) {
+      a.lvn[((int64_t)c * nlev + i) * a.N + n] = 0u;
+      a.lvq[((int64_t)c * nlev + i) * a.N + n] = 0ull;
+    }
+  }
+  const DevPolicy P = a.pol[c];
+  const HT hmask = P.H >= (int)(8 * sizeof(HT)) ? (HT)~(HT)0 : (HT)(((HT)1 << P.H) - 1);
+  const int32_t t0 = s * a.seg_len, t1 = min(a.T, t0 + a.seg_len);
+  const int K = lmax - lmin;
+  const int step = (P.variant & MAGUS_VARIANT_GRADUAL) ? P.step : K;
+  HT hist = (HT)history_at(a, P, n, max(t0, P.W)) & hmask;
+  int d = 0, lo = lmin, hi = lmax;  // identity
+  uint32_t* mk = a.mask + (int64_t)cl * 3 * a.nw * a.N + n;
+  const int ld32 = (int)a.ld;
+  uint32_t inc = 0, dcr = 0, hw = 0;
+  // one round: Alg. 2, Alg. 1, the event log, and the composition with this
+  // round's map: hold, +-step (l.18 / l.23-25), or the override to max (l.10)
+  auto round = [&](int i, float xt, float xl) {
+    const double D = (double)xt - (double)xl;
+    const bool pi = D > P.d_inc, pd = !pi && D < P.d_dec;
+    const bool hf = __popc((uint32_t)(hist & hmask)) + (sizeof(HT) > 4 ? __popc((uint32_t)((uint64_t)hist >> 32)) : 0) >= P.k;
+    inc |= (uint32_t)pi << i;
+    dcr |= (uint32_t)pd << i;
+    hw |= (uint32_t)hf << i;
+    hist = ((hist << 1) | (HT)(pi || pd)) & hmask;
+    const int sd = pi ? step : (pd ? -step : 0);
+    const int nd = min(max(d + sd, -K), K);
+    const int nlo = min(max(lo + sd, lmin), lmax), nhi = min(max(hi + sd, lmin), lmax);
+    d = hf ? 0 : nd;
+    lo = hf ? lmax : nlo;
+    hi = hf ? lmax : nhi;
+  };
+  for (int32_t tw = t0; tw < t1; tw += 32) {
+    inc = dcr = hw = 0;
+    if (tw >= P.W && tw + 32 <= t1) {   // a full word of MDFS rounds
+      const float* px = a.x + (int64_t)tw * a.ld + n;
+      const float* pl = px - (int64_t)(P.W - 1) * a.ld;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        float xs[kWalkChunk], xl[kWalkChunk];
+        load16(px + h * kWalkChunk * ld32, ld32, xs);
+        load16(pl + h * kWalkChunk * ld32, ld32, xl);
+#pragma unroll
+        for (int i = 0; i < kWalkChunk; ++i) round(h * kWalkChunk + i, xs[i], xl[i]);
+      }
+    } else {                            // warm-up rounds (t < W) / the ragged tail
+      for (int32_t t = max(tw, P.W); t < min(tw + 32, t1); ++t)
+        round(t - tw, a.x[(int64_t)t * a.ld + n], a.x[(int64_t)(t - P.W + 1) * a.ld + n]);
+    }
+    const int64_t w = tw >> 5;
+    mk[w * a.N] = inc;
+    mk[(a.nw + w) * a.N] = dcr;
+    mk[(2 * (int64_t)a.nw + w) * a.N] = hw;
+  }
+  if (s < a.nseg - 1) a.map[((int64_t)cl * a.nseg + s) * a.N + n] = map_pack(d, lo, hi);
+}
+
+// Pass 2: the same threads replay the step rule from the true carry-in and
+// meter model M at the level that governs each interval.
+__global__ void __launch_bounds__(kWalkThreads, 4) walk_replay_kernel(WalkArgs a, DevPlatform plat,
+                                                                   const __grid_constant__ WalkLevels lv) {
+  __shared__ double s_invB[kWalkMaxLv];
+  __shared__ float s_xthr[kWalkMaxLv];
+  __shared__ uint8_t s_bkeep[kWalkMaxLv];
+  const int lmin = plat.r_min, lmax = plat.r_max, nlev = lmax - lmin + 1;
+  for (int i = threadIdx.x; i < nlev; i += kWalkThreads) {
+    s_invB[i] = lv.invB[i];
+    s_xthr[i] = lv.xthr[i];
+    s_bkeep[i] = lv.bkeep[i];
+  }
+  __syncthreads();
+  const int64_t n = (int64_t)blockIdx.x * kWalkThreads + threadIdx.x;
+  const int32_t s = blockIdx.y, cl = blockIdx.z, c = a.c0 + cl;
+  if (n >= a.N) return;
+  const DevPolicy P = a.pol[c];
+  const int32_t t0 = s * a.seg_len, t1 = min(a.T, t0 + a.seg_len);
+  const int step = (P.variant & MAGUS_VARIANT_GRADUAL) ? P.step : (lmax - lmin);
+
+  // carry-in dec[t0 - 1]: dec[-1] := r_max (P@23755), then every earlier
+  // segment's map
+  int lvl = lmax;
+  for (int32_t j = 0; j < s; ++j) lvl = map_apply(a.map[((int64_t)cl * a.nseg + j) * a.N + n], lvl);
+
+  int cur = lvl;                       // level of the current run of intervals (= dec[t-1])
+  int32_t run_start = t0;
+  unsigned long long run_q = 0;
+  double invB_cur = s_invB[cur - lmin];
+  float xthr_cur = s_xthr[cur - lmin];
+  int bkeep_cur = s_bkeep[cur - lmin];
+  int32_t events = 0, hi_rounds = 0, msr = 0, changes = 0, n_min_dec = 0, b_base = 0, b_magus = 0;
+  unsigned long long q_base = 0, digest = 0;
+  const bool bursts = plat.burst_on != 0;
+  const double invB_max = plat.invB_max;
+  const float xthr_max = plat.xthr_max, xburst = plat.xburst;
+  unsigned int* lvn = a.lvn + (int64_t)c * nlev * a.N + n;
+  unsigned long long* lvq = a.lvq + (int64_t)c * nlev * a.N + n;
+  const uint32_t* mk = a.mask + (int64_t)cl * 3 * a.nw * a.N + n;
+  const int ld32 = (int)a.ld;
+  uint32_t inc = 0, dcr = 0, hw = 0, word = 0;
+
+  // interval t (at cur), then round t's decision from the pass-1 masks
+  // (all zero in the warm-up, t < W)
+  auto interval = [&](int i, int32_t t, float xt) {
+    if (xt > xthr_cur) run_q += q_literal(xt, invB_cur);       // model M stretch at dec[t-1]
+    if (xt > xthr_max) q_base += q_literal(xt, invB_max);      // ... and at r_max
+    if (bursts && xt > xburst) {                               // Sec. 6.3 bursts
+      ++b_base;
+      b_magus += bkeep_cur;
+    }
+    const bool hf = (hw >> i) & 1u, pi = (inc >> i) & 1u, pd = (dcr >> i) & 1u;
+    const int sd = pi ? step : (pd ? -step : 0);
+    const int nl = min(max(lvl + sd, lmin), lmax);
+    lvl = hf ? lmax : nl;                                      // l.10 / l.18-19 / l.23-25
+    word |= (uint32_t)(lvl == lmin) << i;
+    if (a.levels) a.levels[((int64_t)c * a.T + t) * a.N + n] = (uint8_t)lvl;
+    if (lvl != cur) {                                          // a change (never at t = 0)
+      ++changes;
+      atomicAdd(lvn + (int64_t)(cur - lmin) * a.N, (unsigned int)(t + 1 - run_start));
+      if (run_q) atomicAdd(lvq + (int64_t)(cur - lmin) * a.N, run_q);
+      run_start = t + 1;
+      run_q = 0;
+      cur = lvl;
+      invB_cur = s_invB[cur - lmin];
+      xthr_cur = s_xthr[cur - lmin];
+      bkeep_cur = s_bkeep[cur - lmin];
+    }
+  };
+  for (int32_t tw = t0; tw < t1; tw += 32) {
+    const int64_t w = tw >> 5;
+    inc = mk[w * a.N];
+    dcr = mk[(a.nw + w) * a.N];
+    hw = mk[(2 * (int64_t)a.nw + w) * a.N];
+    events += __popc(inc | dcr);                               // l.17 / l.22
+    hi_rounds += __popc(hw);
+    msr += __popc(inc | dcr | hw);                             // tune_uncore_freq calls
+    word = 0;
+    if (tw + 32 <= t1) {
+      const float* px = a.x + (int64_t)tw * a.ld + n;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        float xs[kWalkChunk];
+        load16(px + h * kWalkChunk * ld32, ld32, xs);
+#pragma unroll
+        for (int i = 0; i < kWalkChunk; ++i) interval(h * kWalkChunk + i, tw + h * kWalkChunk + i, xs[i]);
+      }
+    } else {
+      for (int32_t t = tw; t < t1; ++t) interval(t - tw, t, a.x[(int64_t)t * a.ld + n]);
+    }
+    n_min_dec += __popc(word);
+    if (a.dec) a.dec[((int64_t)c * a.nw + w) * a.N + n] = word;
+    digest += (unsigned long long)word * digest_mul(w);
+  }
+  atomicAdd(lvn + (int64_t)(cur - lmin) * a.N, (unsigned int)(t1 - run_start));
+  if (run_q) atomicAdd(lvq + (int64_t)(cur - lmin) * a.N, run_q);
+  unsigned long long* acc = a.acc + (int64_t)c * kWalkFields * a.N + n;
+  const unsigned long long vals[kWalkFields] = {
+      (unsigned long long)events, (unsigned long long)hi_rounds, (unsigned long long)msr,
+      (unsigned long long)changes, (unsigned long long)n_min_dec, q_base, digest,
+      (unsigned long long)b_base, (unsigned long long)b_magus};
+#pragma unroll
+  for (int f = 0; f < kWalkFields; ++f)
+    if (vals[f]) atomicAdd(acc + (int64_t)f * a.N, vals[f]);
+}
+
+__global__ void __launch_bounds__(kWalkThreads) walk_final_kernel(WalkArgs a, DevPlatform plat) {
+  const int64_t gid = (int64_t)blockIdx.x * kWalkThreads + threadIdx.x;
+  if (gid >= a.N * a.C) return;
+  const int32_t c = (int32_t)(gid / a.N);
+  const int64_t n = gid - (int64_t)c * a.N;
+  const int lmin = plat.r_min, lmax = plat.r_max, nlev = lmax - lmin + 1;
+  const unsigned long long* acc = a.acc + (int64_t)c * kWalkFields * a.N + n;
+  const unsigned int* lvn = a.lvn + (int64_t)c * nlev * a.N + n;
+  const unsigned long long* lvq = a.lvq + (int64_t)c * nlev * a.N + n;
+  const int64_t n_min_int = lvn[0];
+  const uint64_t q_min = lvq[0];
+  uint64_t q_max = 0;
+  for (int i = 1; i < nlev; ++i) q_max += lvq[(int64_t)i * a.N];
+  magus_summary* so = a.summary + gid;
+  magus_base* bo = (a.base && c == 0) ? a.base + n : nullptr;
+  const int64_t changes = (int64_t)acc[WF_CH * a.N];
+  finalize_summary(plat, a.T, (int64_t)acc[WF_EV * a.N], (int64_t)acc[WF_HI * a.N], (int64_t)acc[WF_MSR * a.N],
+                   changes, (int64_t)acc[WF_MDEC * a.N], n_min_int, q_min, q_max, acc[WF_QBASE * a.N],
+                   acc[WF_DIG * a.N], (int64_t)acc[WF_BB * a.N], (int64_t)acc[WF_BM * a.N], so, bo);
+  // general model M: energy = sum over the ratios, ascending
+  double energy = 0.0;
+  for (int i = 0; i < nlev; ++i) {
+    const int l = lmin + i;
+    const double Pl = a.p_lo + (a.p_span * (double)(l - lmin)) / (double)(lmax - lmin);
+    energy = energy + Pl * (plat.dt * (double)lvn[(int64_t)i * a.N] + plat.cQ * (double)lvq[(int64_t)i * a.N]);
+  }
+  so->energy_j = energy + plat.e_sw * (double)changes;
+}
+
+}  // namespace
+
+// configs per launch: the pass-1 masks of a batch stay below this
+constexpr size_t kWalkMaskBudget = size_t(1) << 30;
+
+static int64_t walk_batch(int64_t N, int32_t C, int64_t T) {
+  const size_t per = 3 * 4 * (size_t)((T + 31) / 32) * (size_t)N;
+  return std::max<int64_t>(1, std::min<int64_t>(C, (int64_t)(kWalkMaskBudget / std::max<size_t>(per, 1))));
+}
+
+size_t walk_scratch_bytes(int64_t N, int32_t C, int64_t T, int64_t nseg, const DevPlatform& plat) {
+  const int nlev = plat.r_max - plat.r_min + 1;
+  const int64_t B = walk_batch(N, C, T), nw = (T + 31) / 32;
+  auto al = [](size_t b) { return (b + 255) / 256 * 256; };
+  return al(4 * (size_t)B * nseg * N) + al(12 * (size_t)B * nw * N) + al(8 * (size_t)C * kWalkFields * N) +
+         al(4 * (size_t)C * nlev * N) + al(8 * (size_t)C * nlev * N);
+}
+
+int launch_walk(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld, const DevPolicy* pol_dev,
+                int32_t C, int32_t max_H, const DevPlatform& plat, double bw_max, double p_lo, double p_span,
+                int64_t nseg, int64_t seg_len, void* scratch, magus_summary* out_summary, magus_base* out_base,
+                uint32_t* out_dec, uint8_t* out_levels) {
+  const int nlev = plat.r_max - plat.r_min + 1;
+  const int64_t B = walk_batch(N, C, T), nw = (T + 31) / 32;
+  auto al = [](size_t b) { return (b + 255) / 256 * 256; };
+  char* sp = (char*)scratch;
+  WalkArgs a;
+  a.x = x;
+  a.N = N;
+  a.ld = ld;
+  a.T = (int32_t)T;
+  a.nw = (int32_t)nw;
+  a.pol = pol_dev;
+  a.C = C;
+  a.c0 = 0;
+  a.nseg = (int32_t)nseg;
+  a.seg_len = (int32_t)seg_len;
+  a.map = (uint32_t*)sp;
+  sp += al(4 * (size_t)B * nseg * N);
+  a.mask = (uint32_t*)sp;
+  sp += al(12 * (size_t)B * nw * N);
+  a.acc = (unsigned long long*)sp;
+  sp += al(8 * (size_t)C * kWalkFields * N);
+  a.lvn = (unsigned int*)sp;
+  sp += al(4 * (size_t)C * nlev * N);
+  a.lvq = (unsigned long long*)sp;
+  a.summary = out_summary;
+  a.base = out_base;
+  a.dec = out_dec;
+  a.levels = out_levels;
+  a.p_lo = p_lo;
+  a.p_span = p_span;
+  // per-level constants: B_l = (bw_max * l) / r_max, 1 / B_l (kernels_ref.cu capacity())
+  WalkLevels lv{};
+  for (int i = 0; i < nlev; ++i) {
+    const int l = plat.r_min + i;
+    const double Bl = (bw_max * (double)l) / (double)plat.r_max;
+    lv.invB[i] = 1.0 / Bl;
+    lv.xthr[i] = stretch_threshold(lv.invB[i]);
+    lv.bkeep[i] = (plat.burst_on && Bl > plat.burst_mbs) ? 1 : 0;
+  }
+  int launched = 0;
+  auto mk = max_H > 32 ? walk_map_kernel<uint64_t> : walk_map_kernel<uint32_t>;
+  for (int64_t c0 = 0; c0 < C; c0 += B) {
+    a.c0 = (int32_t)c0;
+    const dim3 grid((unsigned)((N + kWalkThreads - 1) / kWalkThreads), (unsigned)nseg,
+                    (unsigned)std::min<int64_t>(B, C - c0));
+    mk<<<grid, kWalkThreads, 0, s>>>(a, plat.r_min, plat.r_max, nlev);
+    walk_replay_kernel<<<grid, kWalkThreads, 0, s>>>(a, plat, lv);
+    launched += 2;
+  }
+  const unsigned fb = (unsigned)((N * C + kWalkThreads - 1) / kWalkThreads);
+  walk_final_kernel<<<fb, kWalkThreads, 0, s>>>(a, plat);
+  return cudaGetLastError() == cudaSuccess ? launched + 1 : -1;
+}
+
+}  // namespace magus

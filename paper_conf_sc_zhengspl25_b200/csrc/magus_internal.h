@@ -112,6 +112,14 @@ int launch_seq(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,
                double p_lo, double p_span, bool closed, bool multi, magus_summary* out_summary,
                magus_base* out_base, uint32_t* out_dec, uint8_t* out_levels);
 
+// Time-segmented open-loop kernel (kernels_walk.cu): f4 and level output;
+// scratch = maps + accumulators (walk_scratch_bytes); out_summary required.
+size_t walk_scratch_bytes(int64_t N, int32_t C, int64_t T, int64_t nseg, const DevPlatform& plat);
+int launch_walk(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld, const DevPolicy* pol_dev,
+                int32_t C, int32_t max_H, const DevPlatform& plat, double bw_max, double p_lo, double p_span,
+                int64_t nseg, int64_t seg_len, void* scratch, magus_summary* out_summary, magus_base* out_base,
+                uint32_t* out_dec, uint8_t* out_levels);
+
 bool stream_supported(int32_t W, int32_t H);
 // Fused stream kernel over nbund bundles of NB configs (bundles_dev:
 // [nbund][NB] global config indices, -1 = padding).  All configs of a launch
