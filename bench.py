@@ -321,7 +321,7 @@ def run_ours(args):
     alg_bytes = N * T * 4 + (C * N * T / 8 if want_dec else 0)
     achieved = alg_bytes / (kern_ms * 1e-3) / 1e9
     traffic = None
-    kname = {1: "ref_kernel", 2: "stream_kernel", 3: "seq_kernel", 4: "walk_replay_kernel"}.get(st["last_kernel"], "?")
+    kname = {1: "ref_kernel", 2: "stream_kernel", 3: "seq_kernel", 4: "walk_map_kernel + walk_replay_kernel + walk_final_kernel"}.get(st["last_kernel"], "?")
     vtag = {0: "", 1: "_f3", 2: "_f4"}.get(args.variant, f"_v{args.variant}")
     # traffic only from an ncu capture of this very kernel and workload
     prof = os.path.join(ROOT, "profiles", f"ncu_cfg{args.config}{vtag}.json")

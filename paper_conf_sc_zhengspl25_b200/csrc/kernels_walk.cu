@@ -97,11 +97,12 @@ __device__ __forceinline__ uint64_t history_at(const WalkArgs& a, const DevPolic
   return hist;
 }
 
-// 16 samples x[t0 + i * ld32 rows] (32-bit row offsets: ld < 2^26, checked
+// K samples x[t0 + i rows] (32-bit row offsets: ld < 2^26, checked
 // by the dispatcher, keeps every address one IMAD from the base)
-__device__ __forceinline__ void load16(const float* __restrict__ p, int ld32, float (&v)[kWalkChunk]) {
+template <int K>
+__device__ __forceinline__ void load_rows(const float* __restrict__ p, int ld32, float (&v)[K]) {
 #pragma unroll
-  for (int i = 0; i < kWalkChunk; ++i) v[i] = __ldg(p + i * ld32);
+  for (int i = 0; i < K; ++i) v[i] = __ldg(p + i * ld32);
 }
 
 // Pass 1: per (trace, segment, config) thread, the rounds of the segment in
@@ -109,7 +110,7 @@ __device__ __forceinline__ void load16(const float* __restrict__ p, int ld32, fl
 // >= t_hi), Alg. 1 (host-inverted thresholds), event logging -- recorded as
 // three bit masks per 32-step word, and composed into the segment's map.
 template <typename HT>
-__global__ void __launch_bounds__(kWalkThreads, 4) walk_map_kernel(WalkArgs a, int32_t lmin, int32_t lmax, int32_t nlev) {
+__global__ void __launch_bounds__(kWalkThreads, 5) walk_map_kernel(WalkArgs a, int32_t lmin, int32_t lmax, int32_t nlev) {
   const int64_t n = (int64_t)blockIdx.x * kWalkThreads + threadIdx.x;
   const int32_t s = blockIdx.y, cl = blockIdx.z, c = a.c0 + cl;
   if (n >= a.N) return;
@@ -126,12 +127,13 @@ __global__ void __launch_bounds__(kWalkThreads, 4) walk_map_kernel(WalkArgs a, i
   const int K = lmax - lmin;
   const int step = (P.variant & MAGUS_VARIANT_GRADUAL) ? P.step : K;
   HT hist = (HT)history_at(a, P, n, max(t0, P.W)) & hmask;
-  int d = 0, lo = lmin, hi = lmax;  // identity
+  int d = 0, lo = lmin, hi = lmax;  // identity (the clamp-shift map l -> min(max(l + d, lo), hi))
   uint32_t* mk = a.mask + (int64_t)cl * 3 * a.nw * a.N + n;
   const int ld32 = (int)a.ld;
   uint32_t inc = 0, dcr = 0, hw = 0;
   // one round: Alg. 2, Alg. 1, the event log, and the composition with this
   // round's map: hold, +-step (l.18 / l.23-25), or the override to max (l.10)
+  // one round: Alg. 2 on the H previous events, Alg. 1, the event log
   auto round = [&](int i, float xt, float xl) {
     const double D = (double)xt - (double)xl;
     const bool pi = D > P.d_inc, pd = !pi && D < P.d_dec;
@@ -140,25 +142,20 @@ __global__ void __launch_bounds__(kWalkThreads, 4) walk_map_kernel(WalkArgs a, i
     dcr |= (uint32_t)pd << i;
     hw |= (uint32_t)hf << i;
     hist = ((hist << 1) | (HT)(pi || pd)) & hmask;
-    const int sd = pi ? step : (pd ? -step : 0);
-    const int nd = min(max(d + sd, -K), K);
-    const int nlo = min(max(lo + sd, lmin), lmax), nhi = min(max(hi + sd, lmin), lmax);
-    d = hf ? 0 : nd;
-    lo = hf ? lmax : nlo;
-    hi = hf ? lmax : nhi;
   };
   for (int32_t tw = t0; tw < t1; tw += 32) {
     inc = dcr = hw = 0;
     if (tw >= P.W && tw + 32 <= t1) {   // a full word of MDFS rounds
       const float* px = a.x + (int64_t)tw * a.ld + n;
       const float* pl = px - (int64_t)(P.W - 1) * a.ld;
+      constexpr int kq = kWalkChunk / 2;  // samples + lags: 16 loads ahead
 #pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        float xs[kWalkChunk], xl[kWalkChunk];
-        load16(px + h * kWalkChunk * ld32, ld32, xs);
-        load16(pl + h * kWalkChunk * ld32, ld32, xl);
+      for (int h = 0; h < 32 / kq; ++h) {
+        float xs[kq], xl[kq];
+        load_rows<kq>(px + h * kq * ld32, ld32, xs);
+        load_rows<kq>(pl + h * kq * ld32, ld32, xl);
 #pragma unroll
-        for (int i = 0; i < kWalkChunk; ++i) round(h * kWalkChunk + i, xs[i], xl[i]);
+        for (int i = 0; i < kq; ++i) round(h * kq + i, xs[i], xl[i]);
       }
     } else {                            // warm-up rounds (t < W) / the ragged tail
       for (int32_t t = max(tw, P.W); t < min(tw + 32, t1); ++t)
@@ -168,17 +165,43 @@ __global__ void __launch_bounds__(kWalkThreads, 4) walk_map_kernel(WalkArgs a, i
     mk[w * a.N] = inc;
     mk[(a.nw + w) * a.N] = dcr;
     mk[(2 * (int64_t)a.nw + w) * a.N] = hw;
+    // compose the word's rounds into the map: everything up to the last
+    // override (l.10) collapses to the constant r_max; after it only the
+    // +-step actions (l.18 / l.23-25) remain, visited sparsely
+    uint32_t acts = inc | dcr;
+    if (hw) {
+      const int j = 31 - __clz(hw);
+      d = 0;
+      lo = hi = lmax;
+      acts = j == 31 ? 0u : acts & (0xFFFFFFFEu << j);
+    }
+    while (acts) {
+      const int i = __ffs(acts) - 1;
+      acts &= acts - 1;
+      const int sd = ((inc >> i) & 1u) ? step : -step;
+      d = min(max(d + sd, -K), K);
+      lo = min(max(lo + sd, lmin), lmax);
+      hi = min(max(hi + sd, lmin), lmax);
+    }
   }
   if (s < a.nseg - 1) a.map[((int64_t)cl * a.nseg + s) * a.N + n] = map_pack(d, lo, hi);
 }
 
 // Pass 2: the same threads replay the step rule from the true carry-in and
-// meter model M at the level that governs each interval.
-__global__ void __launch_bounds__(kWalkThreads, 4) walk_replay_kernel(WalkArgs a, DevPlatform plat,
+// meter model M at the level that governs each interval.  Per round only
+// the level walk and three bit masks (decision at r_min, level change,
+// sample above the capacity at r_min -- a superset of every level's stretch
+// since B_l grows with l -- and bursts) are on the per-sample path; the
+// word's levels go to shared memory, and the sparse work (stretch q at the
+// level of each flagged interval, per-level run lengths at each change,
+// burst counts) runs once per word over the set bits.
+template <bool BURST>
+__global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a, DevPlatform plat,
                                                                    const __grid_constant__ WalkLevels lv) {
   __shared__ double s_invB[kWalkMaxLv];
   __shared__ float s_xthr[kWalkMaxLv];
   __shared__ uint8_t s_bkeep[kWalkMaxLv];
+  __shared__ uint8_t s_lv[32][kWalkThreads];  // dec[32w + i] of the current word
   const int lmin = plat.r_min, lmax = plat.r_max, nlev = lmax - lmin + 1;
   for (int i = threadIdx.x; i < nlev; i += kWalkThreads) {
     s_invB[i] = lv.invB[i];
@@ -186,7 +209,8 @@ __global__ void __launch_bounds__(kWalkThreads, 4) walk_replay_kernel(WalkArgs a
     s_bkeep[i] = lv.bkeep[i];
   }
   __syncthreads();
-  const int64_t n = (int64_t)blockIdx.x * kWalkThreads + threadIdx.x;
+  const int tid = threadIdx.x;
+  const int64_t n = (int64_t)blockIdx.x * kWalkThreads + tid;
   const int32_t s = blockIdx.y, cl = blockIdx.z, c = a.c0 + cl;
   if (n >= a.N) return;
   const DevPolicy P = a.pol[c];
@@ -198,49 +222,33 @@ __global__ void __launch_bounds__(kWalkThreads, 4) walk_replay_kernel(WalkArgs a
   int lvl = lmax;
   for (int32_t j = 0; j < s; ++j) lvl = map_apply(a.map[((int64_t)cl * a.nseg + j) * a.N + n], lvl);
 
-  int cur = lvl;                       // level of the current run of intervals (= dec[t-1])
+  int cur = lvl;                       // level of the current run of intervals
   int32_t run_start = t0;
-  unsigned long long run_q = 0;
-  double invB_cur = s_invB[cur - lmin];
-  float xthr_cur = s_xthr[cur - lmin];
-  int bkeep_cur = s_bkeep[cur - lmin];
+  int qlev = lvl;                      // stretch q of level qlev not yet flushed
+  unsigned long long qacc = 0;
   int32_t events = 0, hi_rounds = 0, msr = 0, changes = 0, n_min_dec = 0, b_base = 0, b_magus = 0;
   unsigned long long q_base = 0, digest = 0;
-  const bool bursts = plat.burst_on != 0;
   const double invB_max = plat.invB_max;
-  const float xthr_max = plat.xthr_max, xburst = plat.xburst;
+  const float xthr_min = plat.xthr_min, xthr_max = plat.xthr_max, xburst = plat.xburst;
   unsigned int* lvn = a.lvn + (int64_t)c * nlev * a.N + n;
   unsigned long long* lvq = a.lvq + (int64_t)c * nlev * a.N + n;
   const uint32_t* mk = a.mask + (int64_t)cl * 3 * a.nw * a.N + n;
   const int ld32 = (int)a.ld;
-  uint32_t inc = 0, dcr = 0, hw = 0, word = 0;
+  uint32_t inc = 0, dcr = 0, hw = 0, word = 0, chg = 0, big = 0, bst = 0;
 
-  // interval t (at cur), then round t's decision from the pass-1 masks
-  // (all zero in the warm-up, t < W)
-  auto interval = [&](int i, int32_t t, float xt) {
-    if (xt > xthr_cur) run_q += q_literal(xt, invB_cur);       // model M stretch at dec[t-1]
-    if (xt > xthr_max) q_base += q_literal(xt, invB_max);      // ... and at r_max
-    if (bursts && xt > xburst) {                               // Sec. 6.3 bursts
-      ++b_base;
-      b_magus += bkeep_cur;
-    }
+  // round i of the word: the step rule from the pass-1 masks (all zero in
+  // the warm-up, t < W), and the per-sample flags of interval 32w + i
+  auto round = [&](int i, float xt) {
+    big |= (uint32_t)(xt > xthr_min) << i;
+    if (BURST) bst |= (uint32_t)(xt > xburst) << i;
     const bool hf = (hw >> i) & 1u, pi = (inc >> i) & 1u, pd = (dcr >> i) & 1u;
     const int sd = pi ? step : (pd ? -step : 0);
     const int nl = min(max(lvl + sd, lmin), lmax);
+    const int prev = lvl;
     lvl = hf ? lmax : nl;                                      // l.10 / l.18-19 / l.23-25
+    s_lv[i][tid] = (uint8_t)lvl;
     word |= (uint32_t)(lvl == lmin) << i;
-    if (a.levels) a.levels[((int64_t)c * a.T + t) * a.N + n] = (uint8_t)lvl;
-    if (lvl != cur) {                                          // a change (never at t = 0)
-      ++changes;
-      atomicAdd(lvn + (int64_t)(cur - lmin) * a.N, (unsigned int)(t + 1 - run_start));
-      if (run_q) atomicAdd(lvq + (int64_t)(cur - lmin) * a.N, run_q);
-      run_start = t + 1;
-      run_q = 0;
-      cur = lvl;
-      invB_cur = s_invB[cur - lmin];
-      xthr_cur = s_xthr[cur - lmin];
-      bkeep_cur = s_bkeep[cur - lmin];
-    }
+    chg |= (uint32_t)(lvl != prev) << i;
   };
   for (int32_t tw = t0; tw < t1; tw += 32) {
     const int64_t w = tw >> 5;
@@ -250,25 +258,63 @@ __global__ void __launch_bounds__(kWalkThreads, 4) walk_replay_kernel(WalkArgs a
     events += __popc(inc | dcr);                               // l.17 / l.22
     hi_rounds += __popc(hw);
     msr += __popc(inc | dcr | hw);                             // tune_uncore_freq calls
-    word = 0;
-    if (tw + 32 <= t1) {
-      const float* px = a.x + (int64_t)tw * a.ld + n;
+    const int before = lvl;                                    // dec[32w - 1]
+    word = chg = big = bst = 0;
+    const int rem = min(32, t1 - tw);
+    const float* px = a.x + (int64_t)tw * a.ld + n;
+    if (rem == 32) {
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
         float xs[kWalkChunk];
-        load16(px + h * kWalkChunk * ld32, ld32, xs);
+        load_rows<kWalkChunk>(px + h * kWalkChunk * ld32, ld32, xs);
 #pragma unroll
-        for (int i = 0; i < kWalkChunk; ++i) interval(h * kWalkChunk + i, tw + h * kWalkChunk + i, xs[i]);
+        for (int i = 0; i < kWalkChunk; ++i) round(h * kWalkChunk + i, xs[i]);
       }
     } else {
-      for (int32_t t = tw; t < t1; ++t) interval(t - tw, t, a.x[(int64_t)t * a.ld + n]);
+      for (int i = 0; i < rem; ++i) round(i, __ldg(px + i * ld32));
     }
     n_min_dec += __popc(word);
+    changes += __popc(chg);                                    // never at t = 0 (dec[-1] := max)
     if (a.dec) a.dec[((int64_t)c * a.nw + w) * a.N + n] = word;
     digest += (unsigned long long)word * digest_mul(w);
+    if (a.levels)
+      for (int i = 0; i < rem; ++i) a.levels[((int64_t)c * a.T + tw + i) * a.N + n] = s_lv[i][tid];
+    // model M at dec[t-1]: stretch of the flagged intervals, bursts
+    uint32_t m = big | bst;
+    while (m) {
+      const int i = __ffs(m) - 1;
+      m &= m - 1;
+      const int L = i ? (int)s_lv[i - 1][tid] : before;
+      const float xt = __ldg(px + i * ld32);
+      if ((big >> i) & 1u) {
+        if (xt > s_xthr[L - lmin]) {
+          if (L != qlev) {
+            if (qacc) atomicAdd(lvq + (int64_t)(qlev - lmin) * a.N, qacc);
+            qacc = 0;
+            qlev = L;
+          }
+          qacc += q_literal(xt, s_invB[L - lmin]);
+        }
+        if (xt > xthr_max) q_base += q_literal(xt, invB_max);
+      }
+      if (BURST && ((bst >> i) & 1u)) {                        // Sec. 6.3 bursts
+        ++b_base;
+        b_magus += s_bkeep[L - lmin];
+      }
+    }
+    // per-level interval counts: a change in round 32w + i ends the run of
+    // intervals that ran at cur
+    m = chg;
+    while (m) {
+      const int i = __ffs(m) - 1;
+      m &= m - 1;
+      atomicAdd(lvn + (int64_t)(cur - lmin) * a.N, (unsigned int)(tw + i + 1 - run_start));
+      run_start = tw + i + 1;
+      cur = s_lv[i][tid];
+    }
   }
   atomicAdd(lvn + (int64_t)(cur - lmin) * a.N, (unsigned int)(t1 - run_start));
-  if (run_q) atomicAdd(lvq + (int64_t)(cur - lmin) * a.N, run_q);
+  if (qacc) atomicAdd(lvq + (int64_t)(qlev - lmin) * a.N, qacc);
   unsigned long long* acc = a.acc + (int64_t)c * kWalkFields * a.N + n;
   const unsigned long long vals[kWalkFields] = {
       (unsigned long long)events, (unsigned long long)hi_rounds, (unsigned long long)msr,
@@ -376,7 +422,8 @@ int launch_walk(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld
     const dim3 grid((unsigned)((N + kWalkThreads - 1) / kWalkThreads), (unsigned)nseg,
                     (unsigned)std::min<int64_t>(B, C - c0));
     mk<<<grid, kWalkThreads, 0, s>>>(a, plat.r_min, plat.r_max, nlev);
-    walk_replay_kernel<<<grid, kWalkThreads, 0, s>>>(a, plat, lv);
+    if (plat.burst_on) walk_replay_kernel<true><<<grid, kWalkThreads, 0, s>>>(a, plat, lv);
+    else walk_replay_kernel<false><<<grid, kWalkThreads, 0, s>>>(a, plat, lv);
     launched += 2;
   }
   const unsigned fb = (unsigned)((N * C + kWalkThreads - 1) / kWalkThreads);
