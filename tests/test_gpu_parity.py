@@ -38,7 +38,7 @@ def ctx():
 
 def to_oracle_policies(pols):
     return oracle.policies([dict(W=p.window, H=p.history, L=p.deriv_len, tau_inc=p.tau_inc,
-                                 tau_dec=p.tau_dec, t_hi=p.t_hi) for p in pols])
+                                 tau_dec=p.tau_dec, t_hi=p.t_hi, variant=p.variant, step=p.step) for p in pols])
 
 
 def run_gpu(ctx, x_np, pols, kernel, segments=0, ld=None, decisions=True):
