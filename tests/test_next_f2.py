@@ -97,8 +97,10 @@ def test_lambda_trades_energy_for_time():
 # ------------------------------- GPU parity --------------------------------
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("full_grid", [False, True])
-def test_gpu_offline_bound_bit_exact(full_grid):
+@pytest.mark.parametrize("full_grid,r_max", [(False, 22), (True, 22), (True, 25), (True, 12), (False, 25)])
+def test_gpu_offline_bound_bit_exact(full_grid, r_max):
+    """Binary and full-grid DPs (15 and 18 ratios: the register-resident
+    kernels; 5 ratios: the generic one) vs the oracle DP, bit for bit."""
     torch = pytest.importorskip("torch")
     magus = pytest.importorskip("paper_conf_sc_zhengspl25_b200")
     N, T = 150, 1777
@@ -106,7 +108,8 @@ def test_gpu_offline_bound_bit_exact(full_grid):
     lams = [0.0, 25.0, 400.0, 1e6]
     plat = magus.platform_preset()
     plat.e_switch_j, plat.t_switch_s = 2.0, 0.004
-    plat_o = oracle.platform(e_sw=2.0, t_sw=0.004)
+    plat.ratio_max = r_max
+    plat_o = oracle.platform(e_sw=2.0, t_sw=0.004, r_max=r_max)
     with magus.Context(device=0, platform=plat) as ctx:
         out = ctx.offline_bound(torch.from_numpy(x).cuda(), lams, full_grid=full_grid)
         torch.cuda.synchronize()
