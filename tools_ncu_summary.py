@@ -63,6 +63,22 @@ def main() -> None:
     res = {"round": a.round, "kernel": kname, "workload": a.workload, "command": a.command,
            "dram_bytes_per_launch": rd + wr, "dram_read_bytes": rd, "dram_write_bytes": wr,
            "alg_bytes_per_launch": a.alg_bytes or None, "metrics": m}
+    if len(rows) > 3:  # several kernels make one replay (e.g. the walk passes): sum their traffic
+        ks = []
+        for r in rows[2:]:
+            d = dict(zip(hdr, r))
+            u = dict(zip(hdr, units))
+
+            def b(name):
+                return float(d[name]) * SCALE.get(u[name], 1.0) if name in d and d[name] else 0.0
+            ks.append({"kernel": d.get("Kernel Name", ""), "time": d.get("gpu__time_duration.sum"),
+                       "time_unit": u.get("gpu__time_duration.sum"),
+                       "dram_bytes": b("dram__bytes_read.sum") + b("dram__bytes_write.sum"),
+                       "warp_instructions": d.get("smsp__inst_executed.sum"),
+                       "issue_active_pct": d.get("smsp__issue_active.avg.pct_of_peak_sustained_active")})
+        res["kernels"] = ks
+        res["dram_bytes_per_launch"] = sum(k["dram_bytes"] for k in ks)
+        res["kernel"] = " + ".join(k["kernel"].split("(")[0] for k in ks)
     # executed-instruction mix and warp-stall reasons from the source page
     try:
         src = ncu(a.rep, "source", ["--print-source", "sass"])

@@ -1,6 +1,7 @@
 set -x
 O=${OUT:-gpurun_out/r1}
 mkdir -p $O
+python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.limit --format=csv > $O/gpu.txt 2>&1
 python bench.py > $O/bench_cfg2.json 2> $O/bench_cfg2.err
 python bench.py --config 3 --steps 20 --warmup 3 > $O/bench_cfg3.json 2> $O/bench_cfg3.err
@@ -16,5 +17,5 @@ ncu --set full --import-source on --clock-control none -k regex:stream_kernel --
 ncu --set full --import-source on --clock-control none -k regex:stream_kernel --launch-skip 12 -c 1 -o $O/prof_cfg3 python bench.py --config 3 --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > $O/ncu_cfg3.log 2>&1
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_cfg2.csv python bench.py --steps 20 --warmup 3 --no-cpu-baseline --no-e2e > /dev/null 2>&1
 ncu --set full --import-source on --clock-control none -k regex:seq_kernel --launch-skip 3 -c 1 -o $O/prof_cfg2_f3 python bench.py --variant 1 --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > $O/ncu_cfg2_f3.log 2>&1
-ncu --set full --import-source on --clock-control none -k regex:seq_kernel --launch-skip 3 -c 1 -o $O/prof_cfg2_f4 python bench.py --variant 2 --step 2 --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > $O/ncu_cfg2_f4.log 2>&1
+ncu --set full --import-source on --clock-control none -k regex:walk_ --launch-skip 9 -c 3 -o $O/prof_cfg2_f4 python bench.py --variant 2 --step 2 --steps 2 --warmup 3 --no-cpu-baseline --no-e2e > $O/ncu_cfg2_f4.log 2>&1
 ls -la $O
