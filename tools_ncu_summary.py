@@ -87,7 +87,9 @@ def main() -> None:
         ops, stalls = collections.Counter(), collections.Counter()
         total = samples = 0
         for r in src[2:]:
-            if len(r) < len(h) or not r[ix["Source"]].strip():
+            if len(r) < len(h) or not r[ix["Source"]].strip() or r == h:
+                continue  # (a multi-kernel report repeats the header per kernel)
+            if not r[ix["Instructions Executed"]].strip().isdigit():
                 continue
             n = int(r[ix["Instructions Executed"]] or 0)
             total += n
