@@ -252,6 +252,10 @@ def run_ours(args):
         ctx.set_option(magus.OPT_SEGMENTS, args.segments)
     if args.bundle:
         ctx.set_option(magus.OPT_BUNDLE, args.bundle)
+    if args.spec_warm:
+        ctx.set_option(magus.OPT_SPEC_WARM, args.spec_warm)
+    if args.kernel:
+        ctx.set_option(magus.OPT_KERNEL, args.kernel)
     id0, _ = mdist.shard(N * world, world, rank)     # weak scaling: N traces per GPU
     x = ctx.gen_traces(seed, N, T, kind=kind, id0=id0)
     torch.cuda.synchronize()
@@ -321,7 +325,7 @@ def run_ours(args):
     alg_bytes = N * T * 4 + (C * N * T / 8 if want_dec else 0)
     achieved = alg_bytes / (kern_ms * 1e-3) / 1e9
     traffic = None
-    kname = {1: "ref_kernel", 2: "stream_kernel", 3: "seq_kernel", 4: "walk_map_kernel + walk_replay_kernel + walk_final_kernel"}.get(st["last_kernel"], "?")
+    kname = {1: "ref_kernel", 2: "stream_kernel", 3: "seq_kernel", 4: "walk_map_kernel + walk_replay_kernel + walk_final_kernel", 5: "spec_kernel + spec_fix_kernel"}.get(st["last_kernel"], "?")
     vtag = {0: "", 1: "_f3", 2: "_f4"}.get(args.variant, f"_v{args.variant}")
     # traffic only from an ncu capture of this very kernel and workload
     prof = os.path.join(ROOT, "profiles", f"ncu_cfg{args.config}{vtag}.json")
@@ -400,7 +404,7 @@ def run_ours(args):
                        "n_configs": C, "decisions_emitted": want_dec, "seed": hex(seed),
                        "l2": f"inputs {N * T * 4 / 1e9:.2f} GB per GPU > 126 MB L2 (no flush needed)",
                        "parallelism": f"traces sharded over {world} GPU(s); 1 all-reduce of int64 totals ({dist_backend(world)})",
-                       "segments": st["last_segments"], "kernel": {1: "reference", 2: "stream", 3: "sequential", 4: "walk"}.get(st["last_kernel"], "?"),
+                       "segments": st["last_segments"], "kernel": {1: "reference", 2: "stream", 3: "sequential", 4: "walk", 5: "spec"}.get(st["last_kernel"], "?"),
                        "variant": args.variant, "step": args.step if args.variant & 2 else 0},
             "roofline": roof,
             "cpu_baseline": cpu, "e2e": e2e,
@@ -663,6 +667,8 @@ def main():
     ap.add_argument("--full-grid", action="store_true", help="f2 over every ratio, not {min, max}")
     ap.add_argument("--variant", type=int, default=0, help="NEXT f3 (1 closed loop) / f4 (2 gradual)")
     ap.add_argument("--step", type=int, default=1, help="ratio step of the gradual variant")
+    ap.add_argument("--spec-warm", type=int, default=0, help="f3 speculation warm-up rounds (0 auto)")
+    ap.add_argument("--kernel", type=int, default=0, help="MAGUS_OPT_KERNEL (0 auto; 5 = speculative f3)")
     ap.add_argument("--burst", type=float, default=0.0,
                     help="NEXT f1: Sec. 6.3 burst threshold (MB/s); > 0 enables the Jaccard counters")
     ap.add_argument("--chunk", type=int, default=0, help="cfg4: intervals per time chunk (0 = fit ~32 GiB)")

@@ -391,17 +391,23 @@ enum {
   MAGUS_OPT_KERNEL = 0,       /* 0 auto, 1 reference (per-sample, the printed
                                  divisions), 2 stream, 3 sequential (per-sample,
                                  latency-optimised: the auto choice for the
-                                 closed loop f3), 4 walk (time-segmented
-                                 open loop: the auto choice for f4 and level
-                                 output; UNSUPPORTED for closed-loop configs) */
+                                 closed loop with the gradual step), 4 walk
+                                 (time-segmented open loop: the auto choice
+                                 for f4 and level output; UNSUPPORTED for
+                                 closed-loop configs), 5 spec (speculatively
+                                 time-segmented closed loop, jump rule,
+                                 W <= 65; opt-in)        */
   MAGUS_OPT_SEGMENTS = 1,     /* 0 auto, else the number of time segments    */
   MAGUS_OPT_TIMING = 2,       /* 1: record CUDA events around the main kernel */
   MAGUS_OPT_WAVES = 3,        /* auto segmentation: 0 (default) = wave model
                                  (segment count minimising the modelled
                                  rounds x segment length), else aim at this
                                  many waves of CTAs                          */
-  MAGUS_OPT_BUNDLE = 4        /* configs per thread sharing Alg. 1/2 work:
+  MAGUS_OPT_BUNDLE = 4,       /* configs per thread sharing Alg. 1/2 work:
                                  0 auto, or force 1, 2 or 4                  */
+  MAGUS_OPT_SPEC_WARM = 5     /* kernel 5: rounds each segment's speculation
+                                 replays before it (0 = auto, min(segment,
+                                 1024)); any value gives the same results   */
 };
 magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value);
 
@@ -412,6 +418,9 @@ typedef struct {
   int64_t last_segments;      /* time segments used by the last replay       */
   int64_t last_kernel;        /* 1 reference, 2 stream, 3 sequential         */
   int64_t last_grid;          /* CTAs of the last main launch                */
+  int64_t last_reruns;        /* kernel 5: segments whose speculation missed
+                                 and were replayed again, in the last replay
+                                 (read with a device sync); else 0           */
 } magus_stats;
 /* Synchronises when timing is on (reads the events). */
 magus_status magus_get_stats(magus_ctx ctx, magus_stats* out);

@@ -24,8 +24,8 @@ OK, ERR_INVALID_ARG, ERR_NOT_INITIALIZED, ERR_CUDA, ERR_NCCL, ERR_OOM, ERR_UNSUP
 POLICY_PAPER_DEFAULT, POLICY_PAPER_PARETO = 0, 1
 PLATFORM_INTEL_A100, PLATFORM_INTEL_MAX1550 = 0, 1
 GEN_MIX, GEN_ADVERSARIAL = 0, 1
-OPT_KERNEL, OPT_SEGMENTS, OPT_TIMING, OPT_WAVES, OPT_BUNDLE = 0, 1, 2, 3, 4
-KERNEL_AUTO, KERNEL_REFERENCE, KERNEL_STREAM, KERNEL_SEQUENTIAL, KERNEL_WALK = 0, 1, 2, 3, 4
+OPT_KERNEL, OPT_SEGMENTS, OPT_TIMING, OPT_WAVES, OPT_BUNDLE, OPT_SPEC_WARM = 0, 1, 2, 3, 4, 5
+KERNEL_AUTO, KERNEL_REFERENCE, KERNEL_STREAM, KERNEL_SEQUENTIAL, KERNEL_WALK, KERNEL_SPEC = 0, 1, 2, 3, 4, 5
 TOT_WORDS = 18
 TOT_NAMES = ["n_traces", "n_viol", "events", "hi_rounds", "msr_writes", "changes", "min_dec",
              "min_int", "qmin_lo", "qmin_hi", "qmax_lo", "qmax_hi", "qbase_lo", "qbase_hi",
@@ -76,7 +76,8 @@ class PlatformConsts(ctypes.Structure):
 class Stats(ctypes.Structure):
     _fields_ = [("launches_total", ctypes.c_int64), ("main_launches", ctypes.c_int64),
                 ("main_ms_total", ctypes.c_double), ("last_segments", ctypes.c_int64),
-                ("last_kernel", ctypes.c_int64), ("last_grid", ctypes.c_int64)]
+                ("last_kernel", ctypes.c_int64), ("last_grid", ctypes.c_int64),
+                ("last_reruns", ctypes.c_int64)]
 
 
 SUMMARY_DT = np.dtype([("n_events", "<i8"), ("n_hi_rounds", "<i8"), ("n_msr_writes", "<i8"),

@@ -120,6 +120,15 @@ int launch_walk(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld
                 int64_t nseg, int64_t seg_len, void* scratch, magus_summary* out_summary, magus_base* out_base,
                 uint32_t* out_dec, uint8_t* out_levels);
 
+// Speculatively time-segmented closed loop (kernels_spec.cu): f3 with the
+// jump rule; scratch = spec_scratch_bytes; out_summary required.
+bool spec_supported(const magus_policy& p);
+size_t spec_scratch_bytes(int64_t N, int32_t C, int64_t nseg);
+int launch_spec(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld, const DevPolicy* pol_dev,
+                int32_t C, bool wide /* some H > 32 or W > 33 */, const DevPlatform& plat, int64_t nseg, int64_t seg_len, int64_t warm, void* scratch,
+                magus_summary* out_summary, magus_base* out_base, uint32_t* out_dec, uint8_t* out_levels,
+                unsigned int** reruns_out);
+
 bool stream_supported(int32_t W, int32_t H);
 // Fused stream kernel over nbund bundles of NB configs (bundles_dev:
 // [nbund][NB] global config indices, -1 = padding).  All configs of a launch

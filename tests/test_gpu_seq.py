@@ -123,11 +123,11 @@ def test_seq_kernel_nan_and_short_traces():
 
 
 def test_seq_kernel_decision_words_through_replay():
-    """magus_replay with closed-loop configs runs the sequential kernel (auto
-    choice) and writes the same decision words as the oracle."""
+    """magus_replay with closed-loop gradual configs runs the sequential
+    kernel (auto choice) and writes the same decision words as the oracle."""
     N, T = 100, 4099
     x = gen.gen_traces(gen.SEEDS[4], N, T)
-    pols = [magus.make_policy(variant=1), magus.make_policy(W=6, variant=1)]
+    pols = [magus.make_policy(variant=1), magus.make_policy(W=6, variant=3, step=14)]
     ref = oracle.replay(x, _opol(pols), want_dec=True)
     xd = torch.from_numpy(np.ascontiguousarray(x)).cuda()
     with magus.Context(device=0) as ctx:
@@ -142,17 +142,19 @@ def test_seq_kernel_decision_words_through_replay():
 
 
 def test_seq_kernel_rejects_unsupported_closed_window():
-    """A closed-loop jump config with W > 64 cannot run on the sequential
-    kernel: forcing it fails loudly, auto falls back to the per-sample kernel."""
+    """A closed-loop jump config with W > 65 runs on neither the sequential
+    nor the speculative kernel: forcing it fails loudly, auto falls back to
+    the per-sample kernel."""
     N, T = 40, 500
     x = gen.gen_traces(gen.SEEDS[1], N, T)
-    pols = [magus.make_policy(W=65, variant=1)]
+    pols = [magus.make_policy(W=66, variant=1)]
     ref = oracle.replay(x, _opol(pols), want_dec=True)
     xd = torch.from_numpy(np.ascontiguousarray(x)).cuda()
     with magus.Context(device=0) as ctx:
-        ctx.set_option(magus.OPT_KERNEL, 3)
-        with pytest.raises(Exception):
-            ctx.replay_levels(xd, pols)
+        for k in (3, 5):
+            ctx.set_option(magus.OPT_KERNEL, k)
+            with pytest.raises(Exception):
+                ctx.replay_levels(xd, pols)
         ctx.set_option(magus.OPT_KERNEL, 0)
         lv, res = ctx.replay_levels(xd, pols)
         torch.cuda.synchronize()
