@@ -646,7 +646,7 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     nseg = std::min<int64_t>(std::max<int64_t>(nseg, 1), 65535);
     seg_len = ((T + nseg - 1) / nseg + 31) / 32 * 32;
     nseg = (T + seg_len - 1) / seg_len;
-    const int64_t warm = ctx->opt_spec_warm > 0 ? ctx->opt_spec_warm : std::min<int64_t>(seg_len, 1024);
+    const int64_t warm = ctx->opt_spec_warm > 0 ? ctx->opt_spec_warm : std::min<int64_t>(seg_len, 1024);  // measured best
     const size_t sum_bytes = out_summary ? 0 : align_up(sizeof(magus_summary) * (size_t)(N * C), 256);
     const size_t base_bytes = (out_base || !out_totals) ? 0 : align_up(sizeof(magus_base) * (size_t)N, 256);
     st = ensure_scratch(ctx, sum_bytes + base_bytes + spec_scratch_bytes(N, C, nseg) + 256);

@@ -51,6 +51,9 @@ struct SpecArgs {
   unsigned long long* f_hist;       // [C][nseg][N] state at t1 of the replay
   unsigned long long* f_ring;
   uint32_t* f_min;
+  unsigned long long* g_hist;       // [C][nseg][N] the same after the retry pass
+  unsigned long long* g_ring;
+  uint32_t* g_min;
   magus_summary* summary;           // [C][N] (required)
   magus_base* base;                 // [N] or NULL
   uint32_t* dec;                    // [C][nw][N] or NULL
@@ -218,6 +221,46 @@ __global__ void __launch_bounds__(kSpecThreads, 4) spec_kernel(SpecArgs a, SpecP
   a.f_min[ix] = st.at_min;
 }
 
+// One parallel retry pass: a segment whose speculation differs from its
+// predecessor's (speculative) final state is replayed from that state.  An
+// isolated miss -- predecessor right, this guess wrong -- becomes exact
+// here instead of in the sequential fix pass.  Reads f_*, writes g_* (and
+// the segment's speculation, partials and outputs when it replays).
+template <typename ST>
+__global__ void __launch_bounds__(kSpecThreads, 4) spec_retry_kernel(SpecArgs a, SpecPlat sp) {
+  const int64_t n = (int64_t)blockIdx.x * kSpecThreads + threadIdx.x;
+  const int32_t s = blockIdx.y, c = blockIdx.z;
+  if (n >= a.N) return;
+  const int64_t ix = ((int64_t)c * a.nseg + s) * a.N + n;
+  const uint32_t sm = a.s_min[ix];
+  bool same = s == 0 || (sm & 2u);
+  SpecState<ST> st{0, 0, false};
+  if (!same) {
+    const int64_t ip = ix - a.N;      // segment s - 1
+    st.hist = (ST)a.f_hist[ip];
+    st.ring = (ST)a.f_ring[ip];
+    st.at_min = a.f_min[ip] != 0;
+    same = (ST)a.s_hist[ix] == st.hist && (ST)a.s_ring[ix] == st.ring && ((sm & 1u) != 0) == st.at_min;
+  }
+  if (same) {
+    a.g_hist[ix] = a.f_hist[ix];
+    a.g_ring[ix] = a.f_ring[ix];
+    a.g_min[ix] = a.f_min[ix];
+    return;
+  }
+  a.s_hist[ix] = (unsigned long long)st.hist;  // the new speculation
+  a.s_ring[ix] = (unsigned long long)st.ring;
+  a.s_min[ix] = st.at_min;
+  const DevPolicy P = a.pol[c];
+  const int32_t t0 = s * a.seg_len, t1 = min(a.T, t0 + a.seg_len);
+  SpecAcc acc{};
+  spec_run<true>(a, sp, P, c, n, t0, t1, st, acc);
+  store_part(a, c, s, n, acc);
+  a.g_hist[ix] = (unsigned long long)st.hist;
+  a.g_ring[ix] = (unsigned long long)st.ring;
+  a.g_min[ix] = st.at_min;
+}
+
 template <typename ST>
 __global__ void __launch_bounds__(kSpecThreads) spec_fix_kernel(SpecArgs a, SpecPlat sp, DevPlatform plat) {
   const int64_t gid = (int64_t)blockIdx.x * kSpecThreads + threadIdx.x;
@@ -226,7 +269,7 @@ __global__ void __launch_bounds__(kSpecThreads) spec_fix_kernel(SpecArgs a, Spec
   const int64_t n = gid - (int64_t)c * a.N;
   const DevPolicy P = a.pol[c];
   const int64_t i0 = (int64_t)c * a.nseg * a.N + n;  // segment 0 is exact
-  SpecState<ST> tr{(ST)a.f_hist[i0], (ST)a.f_ring[i0], a.f_min[i0] != 0};
+  SpecState<ST> tr{(ST)a.g_hist[i0], (ST)a.g_ring[i0], a.g_min[i0] != 0};
   unsigned int reruns = 0;
   for (int32_t s = 1; s < a.nseg; ++s) {
     const int64_t ix = ((int64_t)c * a.nseg + s) * a.N + n;
@@ -234,9 +277,9 @@ __global__ void __launch_bounds__(kSpecThreads) spec_fix_kernel(SpecArgs a, Spec
     const bool ok = (sm & 2u) || ((ST)a.s_hist[ix] == tr.hist && (ST)a.s_ring[ix] == tr.ring &&
                                   ((sm & 1u) != 0) == tr.at_min);
     if (ok) {
-      tr.hist = (ST)a.f_hist[ix];
-      tr.ring = (ST)a.f_ring[ix];
-      tr.at_min = a.f_min[ix] != 0;
+      tr.hist = (ST)a.g_hist[ix];
+      tr.ring = (ST)a.g_ring[ix];
+      tr.at_min = a.g_min[ix] != 0;
     } else {                          // replay the segment from the true state
       const int32_t t0 = s * a.seg_len, t1 = min(a.T, t0 + a.seg_len);
       SpecAcc acc{};
@@ -269,7 +312,7 @@ bool spec_supported(const magus_policy& p) {
 size_t spec_scratch_bytes(int64_t N, int32_t C, int64_t nseg) {
   auto al = [](size_t b) { return (b + 255) / 256 * 256; };
   const size_t cs = (size_t)C * nseg * N;
-  return al(8 * cs * kSpecFields) + 4 * al(8 * cs) + 2 * al(4 * cs) + 256;
+  return al(8 * cs * kSpecFields) + 6 * al(8 * cs) + 3 * al(4 * cs) + 256;
 }
 
 int launch_spec(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld, const DevPolicy* pol_dev,
@@ -304,6 +347,12 @@ int launch_spec(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld
   sc += al(4 * cs);
   a.f_min = (uint32_t*)sc;
   sc += al(4 * cs);
+  a.g_hist = (unsigned long long*)sc;
+  sc += al(8 * cs);
+  a.g_ring = (unsigned long long*)sc;
+  sc += al(8 * cs);
+  a.g_min = (uint32_t*)sc;
+  sc += al(4 * cs);
   a.reruns = (unsigned int*)sc;
   if (reruns_out) *reruns_out = a.reruns;
   a.summary = out_summary;
@@ -329,12 +378,14 @@ int launch_spec(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld
   const unsigned fb = (unsigned)((N * C + kSpecThreads - 1) / kSpecThreads);
   if (wide) {
     spec_kernel<uint64_t><<<grid, kSpecThreads, 0, s>>>(a, sp);
+    spec_retry_kernel<uint64_t><<<grid, kSpecThreads, 0, s>>>(a, sp);
     spec_fix_kernel<uint64_t><<<fb, kSpecThreads, 0, s>>>(a, sp, plat);
   } else {
     spec_kernel<uint32_t><<<grid, kSpecThreads, 0, s>>>(a, sp);
+    spec_retry_kernel<uint32_t><<<grid, kSpecThreads, 0, s>>>(a, sp);
     spec_fix_kernel<uint32_t><<<fb, kSpecThreads, 0, s>>>(a, sp, plat);
   }
-  return cudaGetLastError() == cudaSuccess ? 2 : -1;
+  return cudaGetLastError() == cudaSuccess ? 3 : -1;
 }
 
 }  // namespace magus
