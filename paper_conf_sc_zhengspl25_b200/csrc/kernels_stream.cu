@@ -34,6 +34,10 @@
 
 #include "device_common.cuh"
 
+#ifndef MAGUS_LOOKBACK_SLEEP
+#define MAGUS_LOOKBACK_SLEEP 32  // ns between polls of a predecessor's segment status
+#endif
+
 namespace magus {
 namespace {
 
@@ -686,7 +690,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
       cin = wk.carry ? (wk.carry[(int64_t)c * N + n] & 1u) : 0u;
       for (int64_t jj = s - 1; jj >= 0; --jj) {
         uint32_t v;
-        while (((v = ld_acquire(status + jj * N)) >> 3) != wk.epoch) __nanosleep(32);
+        while (((v = ld_acquire(status + jj * N)) >> 3) != wk.epoch) __nanosleep(MAGUS_LOOKBACK_SLEEP);
         if (v & 2u) { cin = (v >> 2) & 1u; break; }
       }
     }
