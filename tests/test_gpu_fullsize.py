@@ -100,3 +100,17 @@ def test_full_config2_gradual_walk_sampled(ctx):
     for i, n in enumerate(sample):
         for c in range(len(pols)):
             assert np.array_equal(dec[c, :, n], oracle.decision_words(ref.dec[c, i], 8)), (n, c)
+
+
+def test_full_config2_gradual_sweep_in_config_batches(ctx):
+    """Eight gradual configs at 4096 x 100,000: their pass-1 masks (1.2 GB)
+    exceed the walk kernels' 1 GB budget, so the configs run in two batches
+    of map + replay launches; sampled traces vs the oracle."""
+    N, T = 4096, 100_000
+    xd = ctx.gen_traces(gen.SEEDS[2], N, T)
+    pols = [magus.make_policy(variant=2, step=st, tau_inc=ti, t_hi=th)
+            for st in (1, 3) for ti in (200.0, 300.0) for th in (0.3, 0.5)]
+    r = ctx.replay(xd, pols, want_decisions=False)
+    torch.cuda.synchronize()
+    assert ctx.stats()["last_kernel"] == magus.KERNEL_WALK
+    _check_sample(ctx, xd, pols, np.array([0, 1, 2047, N - 1]), r)
