@@ -140,8 +140,39 @@ def dist_env():
     return world, rank, local
 
 
-def cpu_oracle_sample(cfg, T, pols_oracle, budget_s, kind, max_traces=None):
-    """Times the oracle, as it stands, on a bounded sample of the workload."""
+def host_cores() -> int:
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+class OraclePool:
+    """The oracle as it stands, run on several host cores at once over a
+    static partition of the traces (traces are independent; the ctypes call
+    releases the GIL, and the C++ replay keeps no shared state)."""
+
+    def __init__(self, threads: int):
+        from concurrent.futures import ThreadPoolExecutor
+        self.threads = max(1, threads)
+        self.ex = ThreadPoolExecutor(self.threads)
+
+    def replay(self, xs, pols):
+        """xs: [T, N] -> per-config summaries [C, N] (trace order kept)."""
+        import oracle
+        N = xs.shape[1]
+        k = max(1, min(self.threads, N))
+        parts = [np.ascontiguousarray(xs[:, i * N // k:(i + 1) * N // k]) for i in range(k)]
+        res = list(self.ex.map(lambda part: oracle.replay(part, pols), parts))
+        return np.concatenate([r.summary for r in res], axis=1)
+
+    def close(self):
+        self.ex.shutdown()
+
+
+def cpu_oracle_sample(cfg, T, pols_oracle, budget_s, kind, max_traces=None, threads=1):
+    """Times the oracle, as it stands, on a bounded sample of the workload,
+    on `threads` host cores (a static partition of the sampled traces)."""
     import gen
     import oracle
     seed = SEED_BASE + cfg
@@ -154,16 +185,20 @@ def cpu_oracle_sample(cfg, T, pols_oracle, budget_s, kind, max_traces=None):
     t = time.perf_counter()
     oracle.replay(xs, pols_oracle)
     per_trace = (time.perf_counter() - t) / probe_n
-    n = max(1, int(budget_s / max(per_trace, 1e-9)))
+    n = max(1, int(budget_s * threads / max(per_trace, 1e-9)))
     if max_traces:
         n = min(n, max_traces)
-    n = min(n, 1024)  # keeps ld (the oracle's stride) in the probed regime
+    n = min(n, 1024 * threads)  # keeps each part's ld (the oracle's stride) in the probed regime
+    n = max(n, min(threads, max_traces or threads))
     xs = gen.gen_traces(seed, n, T, kind=kind)
+    pool = OraclePool(threads)
+    pool.replay(xs[:64, :pool.threads], pols_oracle)  # threads started, library loaded
     t = time.perf_counter()
-    ref = oracle.replay(xs, pols_oracle)
+    summ = pool.replay(xs, pols_oracle)
     dt = time.perf_counter() - t
+    pool.close()
     units = n * T * len(pols_oracle)
-    return units / dt, n, dt, ref
+    return units / dt, n, dt, summ
 
 
 def policies_for(grid):
@@ -192,23 +227,29 @@ def run_reference(args):
     import oracle
     pols = oracle_policies(policies_for(grid))
     seed = SEED_BASE + args.config
-    per_step = max(1, min(N, 4 if args.config not in (4, 5) else 1))
+    threads = args.cpu_threads or host_cores()
+    per_thread = 4 if args.config not in (4, 5) else 1
+    per_step = max(1, min(N, per_thread * threads))
     xs = gen.gen_traces(seed, per_step, T, kind=kind)
     if args.config in (3, 4):
         pols = pols[:16]  # bounded: 16 of the 256 / 64 configs per step
+    pool = OraclePool(threads)
     for _ in range(args.warmup):
-        oracle.replay(xs, pols)
+        pool.replay(xs, pols)
     t = time.perf_counter()
     for _ in range(args.steps):
-        oracle.replay(xs, pols)
+        pool.replay(xs, pols)
     dt = (time.perf_counter() - t) / args.steps
+    pool.close()
+    cores = min(threads, per_step)
     value = per_step * T * len(pols) / dt
-    sample = f"{per_step} trace(s) x {T} intervals x {len(pols)} config(s) per step (seed {seed:#x})"
+    sample = (f"{per_step} trace(s) x {T} intervals x {len(pols)} config(s) per step (seed {seed:#x}), "
+              f"statically partitioned over {cores} host thread(s)")
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": desc, "n_steps": T, "n_configs": len(pols), "kind": kind},
-            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -368,15 +409,17 @@ def run_ours(args):
         pol_o = oracle_policies(pols)
         if C > 16:
             pol_o = pol_o[:16]
-        v, n_s, dt_s, ref = cpu_oracle_sample(args.config, T, pol_o, args.cpu_budget, kind, max_traces=N)
-        cpu = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"first {n_s} traces x {T} intervals x {len(pol_o)} config(s) of the same workload "
-                         f"({dt_s:.1f} s single-threaded)"}
+        threads = args.cpu_threads or host_cores()
+        v, n_s, dt_s, ref_summ = cpu_oracle_sample(args.config, T, pol_o, args.cpu_budget, kind, max_traces=N,
+                                                   threads=threads)
+        cpu = {"value": v, "unit": UNIT, "cores": min(threads, n_s), "kind": "oracle",
+               "sample": f"first {n_s} traces x {T} intervals x {len(pol_o)} config(s) of the same workload, "
+                         f"statically partitioned over {min(threads, n_s)} host thread(s) ({dt_s:.1f} s)"}
         # parity of that sample against the GPU path (untimed)
         r = ctx.replay(x[:, :n_s], pols[:len(pol_o)], n_traces=n_s, want_totals=False)
         torch.cuda.synchronize()
         got = r.summary_numpy()
-        parity = bool(all(np.array_equal(got[g], ref.summary[o]) for g, o in
+        parity = bool(all(np.array_equal(got[g], ref_summ[o]) for g, o in
                           [("n_events", "n_events"), ("n_changes", "n_changes"), ("digest", "digest"),
                            ("energy_j", "energy"), ("time_s", "time")]))
 
@@ -536,10 +579,12 @@ def run_fleet(args):
     if rank == 0 and not args.no_cpu_baseline:
         import oracle
         pol_o = oracle_policies(pols)[:16]
-        v, n_s, dt_s, ref = cpu_oracle_sample(4, T, pol_o, args.cpu_budget, kind, max_traces=64)
-        cpu = {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"first {n_s} traces x {T} intervals x {len(pol_o)} configs of the fleet "
-                         f"({dt_s:.1f} s single-threaded)"}
+        threads = args.cpu_threads or host_cores()
+        v, n_s, dt_s, ref_summ = cpu_oracle_sample(4, T, pol_o, args.cpu_budget, kind, max_traces=64,
+                                                   threads=threads)
+        cpu = {"value": v, "unit": UNIT, "cores": min(threads, n_s), "kind": "oracle",
+               "sample": f"first {n_s} traces x {T} intervals x {len(pol_o)} configs of the fleet, "
+                         f"statically partitioned over {min(threads, n_s)} host thread(s) ({dt_s:.1f} s)"}
         if world == 1:
             ld_s = (n_s + 3) // 4 * 4
             sb = torch.empty((halo + R, ld_s), dtype=torch.float32, device=dev)
@@ -555,7 +600,7 @@ def run_fleet(args):
                                       want_summary=i == len(chunks) - 1, want_base=False, want_totals=False)
             torch.cuda.synchronize()
             got = r.summary_numpy()
-            parity = bool(all(np.array_equal(got[g], ref.summary[o]) for g, o in
+            parity = bool(all(np.array_equal(got[g], ref_summ[o]) for g, o in
                               [("n_events", "n_events"), ("n_changes", "n_changes"), ("digest", "digest"),
                                ("energy_j", "energy"), ("time_s", "time")]))
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -669,6 +714,7 @@ def main():
     ap.add_argument("--step", type=int, default=1, help="ratio step of the gradual variant")
     ap.add_argument("--spec-warm", type=int, default=0, help="f3 speculation warm-up rounds (0 auto)")
     ap.add_argument("--kernel", type=int, default=0, help="MAGUS_OPT_KERNEL (0 auto; 5 = speculative f3)")
+    ap.add_argument("--cpu-threads", type=int, default=0, help="host threads of the oracle legs (0 = all cores)")
     ap.add_argument("--burst", type=float, default=0.0,
                     help="NEXT f1: Sec. 6.3 burst threshold (MB/s); > 0 enables the Jaccard counters")
     ap.add_argument("--chunk", type=int, default=0, help="cfg4: intervals per time chunk (0 = fit ~32 GiB)")
