@@ -1,0 +1,49 @@
+"""bench.py's contract on the CPU: the reference arm (the oracle on the host
+cores) prints one JSON line with the keys the driver reads, and the
+thread-partitioned oracle used by the CPU baseline equals the plain
+single-threaded oracle trace for trace."""
+from __future__ import annotations
+
+import json
+import os
+import subprocess
+import sys
+
+import numpy as np
+
+import gen
+import oracle
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import bench  # noqa: E402
+
+
+def test_reference_arm_json_line():
+    r = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--steps", "1", "--warmup", "1",
+                        "--cpu-threads", "2"], cwd=ROOT, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stderr
+    lines = [ln for ln in r.stdout.splitlines() if ln.strip()]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    for k in ("impl", "metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step",
+              "higher_is_better", "config", "cpu_baseline", "e2e"):
+        assert k in d, k
+    assert d["impl"] == "reference" and d["value"] > 0 and d["higher_is_better"] is True
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] == 2
+    assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
+    assert d["config"]["workload"].startswith("cfg2")
+
+
+def test_partitioned_oracle_equals_single_thread():
+    x = gen.gen_traces(gen.SEEDS[2], 37, 3000)
+    pols = bench.oracle_policies(bench.policies_for("sweep256"))[:5]
+    ref = oracle.replay(x, pols).summary
+    pool = bench.OraclePool(4)
+    try:
+        got = pool.replay(x, pols)
+    finally:
+        pool.close()
+    assert got.shape == ref.shape
+    for f in ref.dtype.names:
+        assert np.array_equal(got[f], ref[f]), f
