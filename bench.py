@@ -189,6 +189,8 @@ def cpu_oracle_sample(cfg, T, pols_oracle, budget_s, kind, max_traces=None, thre
     if max_traces:
         n = min(n, max_traces)
     n = min(n, 1024 * threads)  # keeps each part's ld (the oracle's stride) in the probed regime
+    if T > 100_000:             # long traces: wide parts stride badly, the probe under-estimates
+        n = min(n, 64 * threads)
     n = max(n, min(threads, max_traces or threads))
     xs = gen.gen_traces(seed, n, T, kind=kind)
     pool = OraclePool(threads)
