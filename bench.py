@@ -279,7 +279,7 @@ def run_ours(args):
     if args.no_decisions:
         want_dec = False
     pols = policies_for(grid)
-    if args.variant:  # NEXT f3 / f4: closed loop / gradual step (per-sample kernel)
+    if args.variant:  # NEXT f3 / f4: closed loop (seq_kernel) / gradual step (walk kernels)
         for p in pols:
             p.variant = args.variant
             p.step = args.step if args.variant & magus.VARIANT_GRADUAL else 0

@@ -78,7 +78,9 @@ typedef struct {
                         throughput min(x_t, B(l_t)) instead of demand (f3);
                         MAGUS_VARIANT_GRADUAL: +-step ratio per event instead
                         of the jump to max/min (f4, the contrast of P@35554).
-                        Non-zero variants run in the per-sample kernel.      */
+                        Non-zero variants run on the sequential (closed
+                        loop) or the time-segmented walk (open loop)
+                        kernels; see MAGUS_OPT_KERNEL.                       */
   int32_t step;      /* ratio step of MAGUS_VARIANT_GRADUAL (>= 1), else 0   */
 } magus_policy;
 enum { MAGUS_VARIANT_CLOSED_LOOP = 1, MAGUS_VARIANT_GRADUAL = 2 };
@@ -267,7 +269,8 @@ magus_status magus_replay_resume(magus_ctx ctx, const float* traces, int64_t n_t
 
 /* Per-interval decisions as uncore ratios (needed for multi-level variants):
  * out_levels DEVICE uint8 [n_params][n_steps][n_traces], level[c][t][n] =
- * dec[t] of trace n under config c.  Runs the per-sample kernel; other
+ * dec[t] of trace n under config c.  Runs the walk kernels (open loop) or
+ * the sequential kernel (closed loop), never the stream kernel; other
  * outputs as in magus_replay.  Asynchronous. */
 magus_status magus_replay_levels(magus_ctx ctx, const float* traces, int64_t n_traces,
                                  int64_t n_steps, int64_t ld, const magus_policy* params,

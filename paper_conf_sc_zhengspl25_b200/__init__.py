@@ -420,7 +420,8 @@ class Context:
 
     def replay_levels(self, traces, policies, n_traces: int | None = None, want_totals: bool = True):
         """Per-interval uncore ratios (uint8 [C, T, N]) + summaries (+ totals):
-        the per-sample kernel, required for the multi-level f4 variant."""
+        walk kernels (open loop) or the sequential kernel (closed loop);
+        required for the multi-level f4 variant."""
         torch = self._torch
         assert traces.is_cuda and traces.dtype == torch.float32 and traces.stride(1) == 1
         T, ld = traces.shape[0], traces.stride(0)

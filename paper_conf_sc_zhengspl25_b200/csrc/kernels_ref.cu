@@ -6,10 +6,11 @@
 // division d = delta / L (P@20631 l.3), event logging (l.17/22/28/31) and
 // the step rule (l.18-25).
 //
-// Roles: (1) the parity baseline of the stream kernel (an independent GPU
-// formulation: literal division, popc of a history register, per-sample
-// accounting); (2) the general fallback (W > 33, H > 32, unaligned traces);
-// (3) the NEXT variants that make the scan truly sequential:
+// Roles: (1) the parity baseline of the stream, sequential, walk and
+// speculative kernels (an independent GPU formulation: literal division,
+// popc of a history register, per-sample accounting); (2) the last-resort
+// fallback (closed-loop configs none of those kernels takes); (3) a literal
+// form of the NEXT variants:
 //   f3 closed loop  -- Alg. 1 observes the delivered throughput
 //                      min(x_t, B(l_t)), which depends on the decision that
 //                      governs interval t, so no time segmentation is exact;
