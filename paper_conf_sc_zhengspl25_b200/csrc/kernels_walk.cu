@@ -202,7 +202,9 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
   __shared__ float s_xthr[kWalkMaxLv];
   __shared__ uint8_t s_bkeep[kWalkMaxLv];
   __shared__ uint8_t s_lv[32][kWalkThreads];  // dec[32w + i] of the current word
+  extern __shared__ unsigned int s_cnt[];     // [nlev][kWalkThreads] intervals per level
   const int lmin = plat.r_min, lmax = plat.r_max, nlev = lmax - lmin + 1;
+  for (int i = 0; i < nlev; ++i) s_cnt[i * kWalkThreads + threadIdx.x] = 0u;
   for (int i = threadIdx.x; i < nlev; i += kWalkThreads) {
     s_invB[i] = lv.invB[i];
     s_xthr[i] = lv.xthr[i];
@@ -224,22 +226,24 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
 
   int cur = lvl;                       // level of the current run of intervals
   int32_t run_start = t0;
+  float xthr_cur = s_xthr[lvl - lmin];  // x > xthr_cur <=> interval t stretches at dec[t-1]
   int qlev = lvl;                      // stretch q of level qlev not yet flushed
   unsigned long long qacc = 0;
   int32_t events = 0, hi_rounds = 0, msr = 0, changes = 0, n_min_dec = 0, b_base = 0, b_magus = 0;
   unsigned long long q_base = 0, digest = 0;
   const double invB_max = plat.invB_max;
-  const float xthr_min = plat.xthr_min, xthr_max = plat.xthr_max, xburst = plat.xburst;
+  const float xthr_max = plat.xthr_max, xburst = plat.xburst;
   unsigned int* lvn = a.lvn + (int64_t)c * nlev * a.N + n;
   unsigned long long* lvq = a.lvq + (int64_t)c * nlev * a.N + n;
   const uint32_t* mk = a.mask + (int64_t)cl * 3 * a.nw * a.N + n;
   const int ld32 = (int)a.ld;
-  uint32_t inc = 0, dcr = 0, hw = 0, word = 0, chg = 0, big = 0, bst = 0;
+  uint32_t inc = 0, dcr = 0, hw = 0, word = 0, chg = 0, big = 0, bmx = 0, bst = 0;
 
   // round i of the word: the step rule from the pass-1 masks (all zero in
   // the warm-up, t < W), and the per-sample flags of interval 32w + i
   auto round = [&](int i, float xt) {
-    big |= (uint32_t)(xt > xthr_min) << i;
+    big |= (uint32_t)(xt > xthr_cur) << i;    // stretched at its level (sparse)
+    bmx |= (uint32_t)(xt > xthr_max) << i;    // ... and at r_max (q_base; rarer still)
     if (BURST) bst |= (uint32_t)(xt > xburst) << i;
     const bool hf = (hw >> i) & 1u, pi = (inc >> i) & 1u, pd = (dcr >> i) & 1u;
     const int sd = pi ? step : (pd ? -step : 0);
@@ -247,6 +251,7 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
     const int prev = lvl;
     lvl = hf ? lmax : nl;                                      // l.10 / l.18-19 / l.23-25
     s_lv[i][tid] = (uint8_t)lvl;
+    xthr_cur = s_xthr[lvl - lmin];
     word |= (uint32_t)(lvl == lmin) << i;
     chg |= (uint32_t)(lvl != prev) << i;
   };
@@ -259,7 +264,7 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
     hi_rounds += __popc(hw);
     msr += __popc(inc | dcr | hw);                             // tune_uncore_freq calls
     const int before = lvl;                                    // dec[32w - 1]
-    word = chg = big = bst = 0;
+    word = chg = big = bmx = bst = 0;
     const int rem = min(32, t1 - tw);
     const float* px = a.x + (int64_t)tw * a.ld + n;
     if (rem == 32) {
@@ -280,23 +285,21 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
     if (a.levels)
       for (int i = 0; i < rem; ++i) a.levels[((int64_t)c * a.T + tw + i) * a.N + n] = s_lv[i][tid];
     // model M at dec[t-1]: stretch of the flagged intervals, bursts
-    uint32_t m = big | bst;
+    uint32_t m = big | bmx | bst;
     while (m) {
       const int i = __ffs(m) - 1;
       m &= m - 1;
       const int L = i ? (int)s_lv[i - 1][tid] : before;
       const float xt = __ldg(px + i * ld32);
       if ((big >> i) & 1u) {
-        if (xt > s_xthr[L - lmin]) {
-          if (L != qlev) {
-            if (qacc) atomicAdd(lvq + (int64_t)(qlev - lmin) * a.N, qacc);
-            qacc = 0;
-            qlev = L;
-          }
-          qacc += q_literal(xt, s_invB[L - lmin]);
+        if (L != qlev) {
+          if (qacc) atomicAdd(lvq + (int64_t)(qlev - lmin) * a.N, qacc);
+          qacc = 0;
+          qlev = L;
         }
-        if (xt > xthr_max) q_base += q_literal(xt, invB_max);
+        qacc += q_literal(xt, s_invB[L - lmin]);
       }
+      if ((bmx >> i) & 1u) q_base += q_literal(xt, invB_max);
       if (BURST && ((bst >> i) & 1u)) {                        // Sec. 6.3 bursts
         ++b_base;
         b_magus += s_bkeep[L - lmin];
@@ -308,12 +311,16 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
     while (m) {
       const int i = __ffs(m) - 1;
       m &= m - 1;
-      atomicAdd(lvn + (int64_t)(cur - lmin) * a.N, (unsigned int)(tw + i + 1 - run_start));
+      s_cnt[(cur - lmin) * kWalkThreads + tid] += (unsigned int)(tw + i + 1 - run_start);
       run_start = tw + i + 1;
       cur = s_lv[i][tid];
     }
   }
-  atomicAdd(lvn + (int64_t)(cur - lmin) * a.N, (unsigned int)(t1 - run_start));
+  s_cnt[(cur - lmin) * kWalkThreads + tid] += (unsigned int)(t1 - run_start);
+  for (int l = 0; l < nlev; ++l) {
+    const unsigned int v = s_cnt[l * kWalkThreads + tid];
+    if (v) atomicAdd(lvn + (int64_t)l * a.N, v);
+  }
   if (qacc) atomicAdd(lvq + (int64_t)(qlev - lmin) * a.N, qacc);
   unsigned long long* acc = a.acc + (int64_t)c * kWalkFields * a.N + n;
   const unsigned long long vals[kWalkFields] = {
@@ -417,13 +424,21 @@ int launch_walk(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld
   }
   int launched = 0;
   auto mk = max_H > 32 ? walk_map_kernel<uint64_t> : walk_map_kernel<uint32_t>;
+  const size_t cnt_smem = (size_t)nlev * kWalkThreads * sizeof(unsigned int);  // <= 65 KB (127 ratios)
+  if (cnt_smem > 48 * 1024) {
+    if (cudaFuncSetAttribute(walk_replay_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cnt_smem) !=
+            cudaSuccess ||
+        cudaFuncSetAttribute(walk_replay_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cnt_smem) !=
+            cudaSuccess)
+      return -1;
+  }
   for (int64_t c0 = 0; c0 < C; c0 += B) {
     a.c0 = (int32_t)c0;
     const dim3 grid((unsigned)((N + kWalkThreads - 1) / kWalkThreads), (unsigned)nseg,
                     (unsigned)std::min<int64_t>(B, C - c0));
     mk<<<grid, kWalkThreads, 0, s>>>(a, plat.r_min, plat.r_max, nlev);
-    if (plat.burst_on) walk_replay_kernel<true><<<grid, kWalkThreads, 0, s>>>(a, plat, lv);
-    else walk_replay_kernel<false><<<grid, kWalkThreads, 0, s>>>(a, plat, lv);
+    if (plat.burst_on) walk_replay_kernel<true><<<grid, kWalkThreads, cnt_smem, s>>>(a, plat, lv);
+    else walk_replay_kernel<false><<<grid, kWalkThreads, cnt_smem, s>>>(a, plat, lv);
     launched += 2;
   }
   const unsigned fb = (unsigned)((N * C + kWalkThreads - 1) / kWalkThreads);
