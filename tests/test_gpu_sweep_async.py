@@ -54,3 +54,26 @@ def test_async_step_matches_sync_step():
         out = ctx.sweep_best_async(r.totals)
         torch.cuda.synchronize()
         assert ctx.sweep_result(out) == ctx.sweep_best(r.totals)
+
+
+@pytest.mark.parametrize("config", [2, 3])
+def test_bench_steps_in_flight_agree(config):
+    """bench.py with two steps in flight (two contexts on two streams)
+    reports the same choice as strictly serial steps, and every launch of
+    both contexts is counted."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    lines = []
+    for inflight in (1, 2):
+        r = subprocess.run([sys.executable, "bench.py", "--config", str(config), "--n-traces", "256", "--n-steps",
+                            "4000", "--steps", "6", "--warmup", "3", "--no-cpu-baseline", "--no-e2e",
+                            "--inflight", str(inflight)], cwd=root, capture_output=True, text=True, timeout=600)
+        assert r.returncode == 0, r.stderr[-2000:]
+        lines.append(json.loads(r.stdout.strip().splitlines()[-1]))
+    a, b = lines
+    assert a["config"]["steps_in_flight"] == 1 and b["config"]["steps_in_flight"] == 2
+    assert a["best_config"] == b["best_config"] and a["feasible"] == b["feasible"]
+    assert a["gpu_launches"] == b["gpu_launches"]
