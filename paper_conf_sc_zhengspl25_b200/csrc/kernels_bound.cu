@@ -101,6 +101,16 @@ bound_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
   o[2] = Tm[b];
 }
 
+// (double)q_literal(x, invB) from the widened sample xd = (double)x, with
+// floor(s * 2^24) formed in fp64 (RZ add of 2^52: exact for 0 < s * 2^24 <=
+// 2^39) -- bit-identical, without an XU conversion per level.
+__device__ __forceinline__ double q_as_double(double xd, double invB) {
+  const double r = xd * invB;
+  double s24 = (r - 1.0 < 32768.0 ? r - 1.0 : 32768.0) * kQScale;
+  s24 = __dsub_rn(__dadd_rz(s24, 4503599627370496.0), 4503599627370496.0);
+  return r > 1.0 ? s24 : 0.0;
+}
+
 // The full ratio grid with a compile-time level count L (the platforms'
 // 15 and 18 ratios): every per-level array is register-resident (fully
 // unrolled loops; the chosen predecessor's energy / time are picked by
@@ -142,8 +152,9 @@ bound_grid_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
       __syncwarp();
     }
     const float xt = s_x[jj][threadIdx.x];
+    const double xd = (double)xt;
     if (t == 0) {
-      const double tau = plat.dt + plat.cQ * (double)q_literal(xt, s_invB[imax]);
+      const double tau = plat.dt + plat.cQ * q_as_double(xd, s_invB[imax]);
       const double e = s_P[imax] * tau;
       V[imax] = e + lam * tau;
       E[imax] = e;
@@ -182,7 +193,7 @@ bound_grid_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
         e0 = sw ? Eo + plat.e_sw : Eo;
         t0 = sw ? To + plat.t_sw : To;
       }
-      const double tau = plat.dt + plat.cQ * (double)q_literal(xt, s_invB[i]);
+      const double tau = plat.dt + plat.cQ * q_as_double(xd, s_invB[i]);
       const double e = s_P[i] * tau;
       V[i] = v + (e + lam * tau);
       E[i] = e0 + e;
@@ -236,8 +247,13 @@ bound_binary_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t l
     for (int i = 0; i < 32; ++i) {
       if (i < rem) {
         const int64_t t = tc + i;
-        const double tau0 = dt + cQ * (double)q_literal(xs[i], invB0);
-        const double tau1 = dt + cQ * (double)q_literal(xs[i], invB1);
+        // model M stretch (q_literal) with the sample widened
+        // once and floor(s * 2^24) formed in fp64 (RZ add of 2^52: exact for
+        // 0 < s * 2^24 <= 2^39), so no XU conversion per level; the value
+        // equals (double)q_literal(x, invB) bit for bit
+        const double xd = (double)xs[i];
+        const double tau0 = dt + cQ * q_as_double(xd, invB0);
+        const double tau1 = dt + cQ * q_as_double(xd, invB1);
         const double e0 = P0 * tau0, e1 = P1 * tau1;
         if (t == 0) {            // interval 0 runs at r_max (reading R6)
           V1 = e1 + lam * tau1;
