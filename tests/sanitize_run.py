@@ -4,7 +4,8 @@ synccheck / initcheck) runs of the TMA + mbarrier + look-back kernels.
   compute-sanitizer --tool racecheck python tests/sanitize_run.py
 
 Exercises: several segments (look-back), a ragged trace group and tail word,
-bundles (NB = 4), bursts, decisions output, the per-sample kernel and the DP.
+bundles (NB = 4), bursts, decisions output, the per-sample kernel, the
+sequential / speculative / walk kernels (level output) and the DP.
 Exits non-zero if the results disagree with the oracle.
 """
 import os
@@ -43,6 +44,30 @@ def main():
             ok &= bool(np.array_equal(got["energy_j"], ref.summary["energy"]))
             ok &= bool(np.array_equal(got["digest"], ref.summary["digest"]))
             ok &= bool(np.array_equal(r.decisions_numpy().transpose(0, 2, 1), oracle.decision_words(ref.dec, 8)))
+        # the sequential (f3), speculative (f3, every guess wrong at warm-up
+        # 1) and walk (f4, several segments) kernels, with level output
+        vpols = [magus.make_policy(variant=1), magus.make_policy(variant=2, step=2),
+                 magus.make_policy(W=5, H=40, variant=2, step=3)]
+        vpo = oracle.policies([dict(W=p.window, H=p.history, L=p.deriv_len, tau_inc=p.tau_inc, tau_dec=p.tau_dec,
+                                    t_hi=p.t_hi, variant=p.variant, step=p.step) for p in vpols])
+        vref = oracle.replay(x, vpo, oracle.platform(burst=12000.0), want_dec=True)
+        runs = [(magus.KERNEL_SEQUENTIAL, vpols[:1], [0], 0),        # f3: seq_kernel<closed, binary>
+                (magus.KERNEL_SEQUENTIAL, vpols, [0, 1, 2], 0),      # mixed: seq_kernel<closed, multi>
+                (magus.KERNEL_SPEC, vpols[:1], [0], 7),
+                (magus.KERNEL_WALK, vpols[1:], [1, 2], 6)]
+        only = os.environ.get("SANITIZE_ONLY")  # e.g. "0,2,3": a subset of the runs above
+        if only:
+            runs = [runs[int(i)] for i in only.split(",")]
+        for kernel, pp, idx, segs in runs:
+            ctx.set_option(magus.OPT_KERNEL, kernel)
+            ctx.set_option(magus.OPT_SEGMENTS, segs)
+            ctx.set_option(magus.OPT_SPEC_WARM, 1)
+            lv, rr = ctx.replay_levels(xd, pp, n_traces=N)
+            torch.cuda.synchronize()
+            ok &= bool(np.array_equal(lv.cpu().numpy().transpose(0, 2, 1), vref.dec[idx].astype(np.uint8)))
+            ok &= bool(np.array_equal(rr.summary_numpy()["energy_j"], vref.summary["energy"][idx]))
+        ctx.set_option(magus.OPT_KERNEL, magus.KERNEL_AUTO)
+        ctx.set_option(magus.OPT_SEGMENTS, 0)
         out = ctx.offline_bound(xd[:200, :8], [0.0, 100.0])
         torch.cuda.synchronize()
         ok &= bool(np.array_equal(out.cpu().numpy()[3, 1], oracle.offline_bound(x[:200, 3], 100.0)))
