@@ -90,10 +90,12 @@ __device__ __forceinline__ void mb_wait(uint32_t bar, uint32_t parity) {
       "r"(parity)
       : "memory");
 }
-// all lanes' shared-memory writes of the word, then one arrival
+// every lane arrives (the slot barriers count 32 arrivals): each lane's own
+// release orders its shared-memory writes of the word before the waiter's
+// acquire (also what compute-sanitizer's racecheck can follow)
 __device__ __forceinline__ void warp_arrive(uint32_t bar) {
   __syncwarp();
-  if ((threadIdx.x & 31) == 0) mb_arrive(bar);
+  mb_arrive(bar);
 }
 
 // delivered throughput of model M at capacity B (oracle `observed`)
@@ -133,7 +135,7 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
   }
   const uint32_t bar0 = sm_addr(s_bar);
   if (threadIdx.x == 0)
-    for (int i = 0; i < 3 * kSlots + kAccountants; ++i) mb_init(bar0 + 8u * i, 1);
+    for (int i = 0; i < 3 * kSlots + kAccountants; ++i) mb_init(bar0 + 8u * i, i < 3 * kSlots ? 32u : 1u);
   __syncthreads();
   // mbarrier addresses (plain arithmetic: no closures on the wait paths)
 #define full(s) (bar0 + 8u * (uint32_t)(s))
