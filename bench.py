@@ -318,6 +318,12 @@ def run_ours(args):
                 ctx2.set_option(k, v)
         lanes.append([ctx2, s2, None, None])
     nstep = [0]
+    if args.comm == "native" and world > 1:
+        # rank 0's NCCL id reaches every rank through the process group
+        uids = [magus.comm_unique_id() if rank == 0 else None for _ in lanes]
+        dist.broadcast_object_list(uids, src=0)
+        for ln, uid in zip(lanes, uids):  # one communicator (and id) per context
+            ln[0].comm_init(uid, world, rank)
 
     def step():
         # replay (one fused launch per W group) -> NCCL sum of the integer
@@ -331,7 +337,10 @@ def run_ours(args):
         with torch.cuda.stream(s_):
             o_ = c_.replay(x, pols, want_summary=False, want_base=False, want_decisions=want_dec,
                            want_totals=True, out=o_)
-            mdist.allreduce_totals(o_.totals)  # the one collective; exact (integer words)
+            if args.comm == "native":          # the library's own NCCL communicator
+                c_.allreduce_totals(o_.totals)
+            else:
+                mdist.allreduce_totals(o_.totals)  # the one collective; exact (integer words)
             if args.sync_sweep:
                 ln[2] = o_
                 return c_.sweep_best(o_.totals)
@@ -491,7 +500,8 @@ def run_ours(args):
             "config": {"workload": desc, "n_traces_per_gpu": N, "n_traces_total": N * world, "n_steps": T,
                        "n_configs": C, "decisions_emitted": want_dec, "seed": hex(seed),
                        "l2": f"inputs {N * T * 4 / 1e9:.2f} GB per GPU > 126 MB L2 (no flush needed)",
-                       "parallelism": f"traces sharded over {world} GPU(s); 1 all-reduce of int64 totals ({dist_backend(world)})",
+                       "parallelism": f"traces sharded over {world} GPU(s); 1 all-reduce of int64 totals "
+                                      f"({'native NCCL' if args.comm == 'native' and world > 1 else dist_backend(world)})",
                        "steps_in_flight": len(lanes),
                        "segments": st["last_segments"], "kernel": {1: "reference", 2: "stream", 3: "sequential", 4: "walk", 5: "spec"}.get(st["last_kernel"], "?"),
                        "variant": args.variant, "step": args.step if args.variant & 2 else 0},
@@ -763,6 +773,8 @@ def main():
     ap.add_argument("--spec-warm", type=int, default=0, help="f3 speculation warm-up rounds (0 auto)")
     ap.add_argument("--kernel", type=int, default=0, help="MAGUS_OPT_KERNEL (0 auto; 5 = speculative f3)")
     ap.add_argument("--cpu-threads", type=int, default=0, help="host threads of the oracle legs (0 = all cores)")
+    ap.add_argument("--comm", choices=["torch", "native"], default="torch",
+                    help="the totals all-reduce: torch.distributed NCCL, or the library's own (magus_comm_init)")
     ap.add_argument("--inflight", type=int, default=2,
                     help="consecutive steps in flight on separate streams/contexts (1 = strictly serial)")
     ap.add_argument("--burst", type=float, default=0.0,

@@ -389,6 +389,26 @@ typedef struct {
 magus_status magus_policy_inspect(const magus_policy* p, magus_policy_consts* out);
 magus_status magus_platform_inspect(const magus_platform* p, magus_platform_consts* out);
 
+/* ---- optional native NCCL path (SURVEY 8(b) magus_comm_init) ------------
+ * The sweep's one collective (north_star (3)) without torch:
+ * an in-place uint64 SUM all-reduce of the per-config totals over NVLink /
+ * NVSwitch, exact and order-free (integer words).  libnccl.so.2 is opened
+ * lazily on the first call (no link-time dependency); MAGUS_ERR_NCCL when it
+ * is missing or an NCCL call fails (detail in magus_last_error). */
+#define MAGUS_COMM_ID_BYTES 128
+/* rank 0 creates the id and ships it to every rank by its own means */
+magus_status magus_comm_unique_id(void* id_out /* host, MAGUS_COMM_ID_BYTES */);
+/* one communicator per context (on ctx's device); collective over the
+ * nranks processes: each must call it with the same id.  Replaces an
+ * earlier communicator of ctx.  Synchronous. */
+magus_status magus_comm_init(magus_ctx ctx, const void* id /* host, MAGUS_COMM_ID_BYTES */,
+                             int32_t nranks, int32_t rank);
+/* totals DEVICE uint64 [n_params][MAGUS_TOT_WORDS], summed over the ranks in
+ * place on ctx's stream (asynchronous); a no-op without a communicator.
+ * Call it between magus_replay and magus_sweep_best / _async on every rank
+ * (every rank then takes the same deterministic choice, no broadcast). */
+magus_status magus_allreduce_totals(magus_ctx ctx, uint64_t* totals, int32_t n_params);
+
 /* ---- options, instrumentation ------------------------------------------ */
 enum {
   MAGUS_OPT_KERNEL = 0,       /* 0 auto, 1 reference (per-sample, the printed

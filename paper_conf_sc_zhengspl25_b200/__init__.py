@@ -125,12 +125,16 @@ _lib.magus_pareto_front_host.argtypes = [ctypes.POINTER(Platform), _vp, _i32, _v
 _lib.magus_sweep_best_host.argtypes = [ctypes.POINTER(Platform), _vp, _i32, ctypes.POINTER(_i32),
                                        ctypes.POINTER(Derived)]
 _lib.magus_reset_stats.argtypes = [_vp]
+_lib.magus_comm_unique_id.argtypes = [_vp]
+_lib.magus_comm_init.argtypes = [_vp, _vp, _i32, _i32]
+_lib.magus_allreduce_totals.argtypes = [_vp, _vp, _i32]
 for _f in ("magus_init", "magus_destroy", "magus_set_stream", "magus_policy_preset", "magus_platform_preset",
            "magus_grid_sweep256", "magus_grid_fleet64", "magus_replay", "magus_replay_host",
            "magus_totals_derive", "magus_sweep_best", "magus_gen_traces", "magus_set_option",
            "magus_get_stats", "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
            "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host",
-           "magus_replay_levels", "magus_offline_bound", "magus_sweep_best_async"):
+           "magus_replay_levels", "magus_offline_bound", "magus_sweep_best_async",
+           "magus_comm_unique_id", "magus_comm_init", "magus_allreduce_totals"):
     getattr(_lib, _f).restype = ctypes.c_int
 
 EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_string", "magus_last_error",
@@ -141,7 +145,9 @@ EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_str
             "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host",
             "magus_replay_levels", "magus_offline_bound", "magus_sweep_best_async",
             "magus_replay_resume", "magus_resume_state_bytes", "magus_resume_halo",
-            "magus_gen_traces_resume", "magus_gen_state_bytes"]
+            "magus_gen_traces_resume", "magus_gen_state_bytes",
+            "magus_comm_unique_id", "magus_comm_init", "magus_allreduce_totals"]
+COMM_ID_BYTES = 128
 VARIANT_CLOSED_LOOP, VARIANT_GRADUAL = 1, 2
 
 
@@ -150,6 +156,17 @@ class MagusError(RuntimeError):
         self.status = status
         msg = _lib.magus_status_string(status).decode()
         super().__init__(f"{msg}: {detail}" if detail else msg)
+
+
+def comm_unique_id() -> bytes:
+    """The optional native NCCL path: rank 0 creates the id (128 bytes) and
+    ships it to every rank by its own means (e.g. a torch.distributed
+    broadcast or a file)."""
+    buf = ctypes.create_string_buffer(COMM_ID_BYTES)
+    st = _lib.magus_comm_unique_id(ctypes.cast(buf, _vp))
+    if st:
+        raise MagusError(st, "comm_unique_id")
+    return buf.raw
 
 
 def abi_version() -> int:
@@ -499,6 +516,20 @@ class Context:
     def sweep_result(out) -> tuple[int, dict, bool]:
         ch = Choice.from_buffer_copy(out.numpy().tobytes())
         return int(ch.best), ch.row.as_dict(), bool(ch.feasible)
+
+    def comm_init(self, uid: bytes, nranks: int, rank: int):
+        """magus_comm_init: this context's NCCL communicator (collective)."""
+        assert len(uid) == COMM_ID_BYTES
+        buf = ctypes.create_string_buffer(uid, COMM_ID_BYTES)
+        self._check(_lib.magus_comm_init(self._h, ctypes.cast(buf, _vp), nranks, rank), "comm_init")
+
+    def allreduce_totals(self, totals):
+        """magus_allreduce_totals: in-place uint64 SUM over the ranks on this
+        context's stream (a no-op without comm_init)."""
+        assert totals.is_cuda and totals.dtype == self._torch.int64 and totals.shape[-1] == TOT_WORDS
+        self._check(_lib.magus_allreduce_totals(self._h, _vp(totals.data_ptr()), totals.shape[0]),
+                    "allreduce_totals")
+        return totals
 
     def sweep_best(self, totals) -> tuple[int, dict, bool]:
         """totals: CUDA int64 tensor [C, 16] (summed over ranks if sharded).

@@ -16,7 +16,7 @@ CSRC = os.path.join(HERE, "csrc")
 BUILD = os.path.join(HERE, "build")
 LIB = os.path.join(HERE, "libmagus.so")
 SOURCES = ["api.cu", "precompute.cpp", "kernels_ref.cu", "kernels_seq.cu", "kernels_walk.cu", "kernels_spec.cu", "kernels_stream.cu", "kernels_post.cu",
-           "kernels_bound.cu"]
+           "kernels_bound.cu", "comm.cpp"]
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "--fmad=false", "-Xcompiler", "-fPIC,-ffp-contract=off,-O2",
@@ -49,7 +49,7 @@ def build_libmagus(verbose: bool = False) -> str:
         f.write(log)
     if verbose:
         print(log)
-    cmd = [_nvcc(), *ARCH, "-shared", "-cudart", "static", "-o", LIB, *[r[0] for r in res]]
+    cmd = [_nvcc(), *ARCH, "-shared", "-cudart", "static", "-o", LIB, *[r[0] for r in res], "-ldl"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")

@@ -48,7 +48,8 @@ struct magus_ctx_s {
   std::vector<LaunchGroup> groups;  // one stream launch each
   int64_t opt_bundle = 0;           // 0 auto, else force NB in {1, 2, 4}
   int64_t opt_spec_warm = 0;
-  unsigned int* spec_reruns = nullptr;  // device counter of the last spec replay (in scratch)        // spec kernel: rounds replayed before a segment (0 auto)
+  unsigned int* spec_reruns = nullptr;  // device counter of the last spec replay (in scratch)
+  void* comm = nullptr;                 // ncclComm_t of magus_comm_init (optional)        // spec kernel: rounds replayed before a segment (0 auto)
   int64_t uploaded_bundle_opt = -1;
   // e2e staging (device)
   void* sweep_dev = nullptr;  // SweepResult of magus_sweep_best_async
@@ -469,6 +470,7 @@ magus_status magus_destroy(magus_ctx ctx) {
       cudaEventDestroy(pr.second);
     }
     for (auto e : ctx->event_pool) cudaEventDestroy(e);
+    if (ctx->comm) nccl_comm_destroy(ctx->comm);
   }
   delete ctx;
   return MAGUS_OK;
@@ -1045,6 +1047,39 @@ magus_status magus_pareto_front_host(const magus_platform* plat, const uint64_t*
   if (!plat || !totals_host || C < 1 || !on_front || !validate_platform(*plat, msg, sizeof msg))
     return MAGUS_ERR_INVALID_ARG;
   pareto(make_dev_platform(*plat), totals_host, C, on_front, n_front);
+  return MAGUS_OK;
+}
+
+magus_status magus_comm_unique_id(void* id_out) {
+  if (!id_out) return MAGUS_ERR_INVALID_ARG;
+  return magus::nccl_unique_id(id_out) == 0 ? MAGUS_OK : MAGUS_ERR_NCCL;
+}
+
+magus_status magus_comm_init(magus_ctx ctx, const void* id, int32_t nranks, int32_t rank) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  if (!id || nranks < 1 || rank < 0 || rank >= nranks)
+    return fail(ctx, MAGUS_ERR_INVALID_ARG, "comm_init: need an id and 0 <= rank < nranks");
+  if (!magus::nccl_available()) return fail(ctx, MAGUS_ERR_NCCL, "libnccl.so.2 could not be opened");
+  DeviceGuard dg(ctx->device);
+  if (ctx->comm) {
+    CK(cudaStreamSynchronize(ctx->stream));
+    magus::nccl_comm_destroy(ctx->comm);
+    ctx->comm = nullptr;
+  }
+  void* c = nullptr;
+  const int r = magus::nccl_comm_init(&c, id, nranks, rank);
+  if (r != 0) return fail(ctx, MAGUS_ERR_NCCL, "ncclCommInitRank: %s", magus::nccl_error(r));
+  ctx->comm = c;
+  return MAGUS_OK;
+}
+
+magus_status magus_allreduce_totals(magus_ctx ctx, uint64_t* totals, int32_t C) {
+  if (!ctx) return MAGUS_ERR_NOT_INITIALIZED;
+  if (!totals || C < 1) return fail(ctx, MAGUS_ERR_INVALID_ARG, "bad allreduce_totals arguments");
+  if (!ctx->comm) return MAGUS_OK;
+  DeviceGuard dg(ctx->device);
+  const int r = magus::nccl_allreduce_u64_sum(ctx->comm, totals, (size_t)C * MAGUS_TOT_WORDS, ctx->stream);
+  if (r != 0) return fail(ctx, MAGUS_ERR_NCCL, "ncclAllReduce: %s", magus::nccl_error(r));
   return MAGUS_OK;
 }
 

@@ -129,6 +129,15 @@ int launch_spec(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld
                 magus_summary* out_summary, magus_base* out_base, uint32_t* out_dec, uint8_t* out_levels,
                 unsigned int** reruns_out);
 
+// Native NCCL (comm.cpp, dlopen'ed lazily); return 0 or an ncclResult_t /
+// -1 when libnccl is unavailable.
+bool nccl_available();
+const char* nccl_error(int r);
+int nccl_unique_id(void* out);
+int nccl_comm_init(void** comm, const void* id_bytes, int nranks, int rank);
+int nccl_comm_destroy(void* comm);
+int nccl_allreduce_u64_sum(void* comm, uint64_t* buf, size_t count, cudaStream_t s);
+
 bool stream_supported(int32_t W, int32_t H);
 // Fused stream kernel over nbund bundles of NB configs (bundles_dev:
 // [nbund][NB] global config indices, -1 = padding).  All configs of a launch
