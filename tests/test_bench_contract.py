@@ -47,3 +47,25 @@ def test_partitioned_oracle_equals_single_thread():
     assert got.shape == ref.shape
     for f in ref.dtype.names:
         assert np.array_equal(got[f], ref[f]), f
+
+
+def test_committed_bench_lines_carry_the_contract_keys():
+    """Every bench line kept under profiles/ has the keys the driver and the
+    judge read (roofline with its fraction, clocks, launches, baselines)."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r01_bench_*.json")))
+    assert files
+    for f in files:
+        d = json.loads(open(f).read().strip().splitlines()[-1])
+        for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better",
+                  "dtype", "data", "config"):
+            assert k in d, (f, k)
+        assert d["value"] > 0, f
+        if d.get("impl") == "reference":
+            assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
+            continue
+        assert "workload" in d["config"], f
+        r = d["roofline"]
+        assert r["bound"] in ("hbm", "alu") and r["peak"] > 0 and r["achieved"] > 0, f
+        assert abs(r["frac"] - r["achieved"] / r["peak"]) < 1e-9, f
+        assert d["gpu_launches"] > 0 and "clocks" in d, f
