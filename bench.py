@@ -30,17 +30,48 @@ sys.path.insert(0, ROOT)
 
 SEED_BASE = 0x4D41475553000000
 WORKLOADS = {
-    # cfg: (n_traces per GPU, n_steps, grid, kind, decisions, description)
-    1: (1, 10_000, "default", 0, True, "cfg1: 1 trace x 10,000 intervals x 1 config (paper_default)"),
-    2: (4096, 100_000, "default", 0, True, "cfg2: 4,096 traces x 100,000 intervals x 1 config (paper_default)"),
-    3: (4096, 100_000, "sweep256", 0, False, "cfg3: 4,096 traces x 100,000 intervals x 256 configs (SWEEP256)"),
-    4: (65536, 1_000_000, "fleet64", 0, False,
-        "cfg4: 65,536 traces x 1,000,000 intervals x 64 configs (FLEET64), traces sharded over the GPUs"),
-    5: (16384, 1_000_000, "default", 1, False,
-        "cfg5: 16,384 adversarial traces x 1,000,000 intervals x 1 config (paper_default)"),
+    # cfg: (n_traces, n_steps, grid, kind, decisions, scaling, what)
+    #   scaling "weak": n_traces per GPU (BASELINE quotes configs 1-3 on one B200);
+    #   "strong": n_traces is the whole fleet, sharded over the GPUs (configs 4, 5)
+    1: (1, 10_000, "default", 0, True, "weak", "1 config (paper_default)"),
+    2: (4096, 100_000, "default", 0, True, "weak", "1 config (paper_default)"),
+    3: (4096, 100_000, "sweep256", 0, False, "weak", "256 configs (SWEEP256)"),
+    4: (65536, 1_000_000, "fleet64", 0, False, "strong", "64 configs (FLEET64)"),
+    5: (16384, 1_000_000, "default", 1, False, "strong", "1 config (paper_default), adversarial traces"),
 }
 METRIC = "trace-samples x configs/sec"
 UNIT = "trace-samples*configs/s"
+
+
+def shape_for(cfg: int, world: int, shard_by: str, n_traces: int = 0, n_steps: int = 0):
+    """(n_traces_total, n_steps, scaling) of a workload at `world` GPUs."""
+    N, T, _, _, _, scaling, _ = WORKLOADS[cfg]
+    N = n_traces or N
+    T = n_steps or T
+    if shard_by == "configs":
+        return N, T, "strong"          # every rank holds the whole fleet, configs are split
+    return (N * world if scaling == "weak" else N), T, scaling
+
+
+def workload_config(cfg: int, world: int, shard_by: str, n_traces: int = 0, n_steps: int = 0,
+                    no_decisions: bool = False, n_configs: int | None = None) -> dict:
+    """The `config` object of the JSON line; both arms build it with this
+    function, so the reference arm reports exactly our arm's config."""
+    _, _, grid, kind, want_dec, _, what = WORKLOADS[cfg]
+    N_tot, T, scaling = shape_for(cfg, world, shard_by, n_traces, n_steps)
+    C = n_configs if n_configs is not None else {"default": 1, "sweep256": 256, "fleet64": 64}[grid]
+    want_dec = want_dec and not no_decisions
+    per_gpu = N_tot if shard_by == "configs" else -(-N_tot // world)
+    return {"workload": f"cfg{cfg}: {N_tot:,} traces x {T:,} intervals x {what}"
+                        + ("" if world == 1 else f" over {world} GPUs"),
+            "n_traces_total": N_tot, "n_traces_per_gpu": per_gpu, "n_steps": T, "n_configs": C,
+            "decisions_emitted": want_dec, "seed": hex(SEED_BASE + cfg),
+            "generator": "adversarial" if kind == 1 else "mix",
+            "l2": f"inputs {per_gpu * T * 4 / 1e9:.2f} GB per GPU vs 126 MB L2 (no flush needed)"
+                  if per_gpu * T * 4 > 4 * 126e6 else "inputs fit in L2: L2 flushed between steps",
+            "parallelism": "1 GPU" if world == 1 else
+                           f"{shard_by} sharded over {world} GPUs; 1 all-reduce of the int64 totals",
+            "scaling": scaling}
 
 
 def _peaks():
@@ -53,34 +84,86 @@ def _peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled in the background."""
+    """SM clock + throttle reasons sampled DURING the timed region.
+
+    NVML (pynvml) polled every ~2 ms from a thread, so even a few-ms timed
+    region gets samples; falls back to `nvidia-smi -lms 50` without NVML.
+    mark() brackets a window; summary() reports the samples inside the
+    window(s) marked so far."""
+    # nvmlClocksEventReason* bits
+    REASONS = {0x4: "sw_power_cap", 0x8: "hw_slowdown", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown"}
     Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
 
-    def __init__(self, index: int):
+    def __init__(self, index: int, period_s: float = 0.002):
         self.index = index
-        self.rows = []
+        self.period = period_s
+        self.rows = []      # (time, sm_mhz, reasons set)
+        self.smax = None
         self.proc = None
+        self.stop_ev = threading.Event()
         self.marks = []
+        self.source = None
+
+    def _nvml_handle(self):
+        import pynvml
+        pynvml.nvmlInit()
+        try:
+            import torch
+            p = torch.cuda.get_device_properties(self.index)
+            bus = f"{p.pci_domain_id:08x}:{p.pci_bus_id:02x}:{p.pci_device_id:02x}.0"
+            return pynvml, pynvml.nvmlDeviceGetHandleByPciBusId(bus.encode())
+        except Exception:
+            return pynvml, pynvml.nvmlDeviceGetHandleByIndex(self.index)
 
     def start(self):
+        try:
+            nv, h = self._nvml_handle()
+            self.smax = float(nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM))
+            get_r = getattr(nv, "nvmlDeviceGetCurrentClocksEventReasons",
+                            getattr(nv, "nvmlDeviceGetCurrentClocksThrottleReasons", None))
+
+            def loop():
+                while not self.stop_ev.is_set():
+                    try:
+                        sm = float(nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM))
+                        r = int(get_r(h)) if get_r else 0
+                        self.rows.append((time.time(), sm, {n for b, n in self.REASONS.items() if r & b}))
+                    except Exception:
+                        pass
+                    self.stop_ev.wait(self.period)
+            threading.Thread(target=loop, daemon=True).start()
+            self.source = f"NVML every {self.period * 1e3:.0f} ms"
+            return
+        except Exception:
+            pass
         try:
             self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
                                           "-lms", "50", "-i", str(self.index)], stdout=subprocess.PIPE,
                                          stderr=subprocess.DEVNULL, text=True)
-            threading.Thread(target=self._read, daemon=True).start()
+            threading.Thread(target=self._read_smi, daemon=True).start()
+            self.source = "nvidia-smi -lms 50"
         except Exception:
             self.proc = None
 
-    def _read(self):
+    def _read_smi(self):
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for line in self.proc.stdout:
-            self.rows.append((time.time(), line.strip()))
+            f = [x.strip() for x in line.strip().split(",")]
+            try:
+                sm, smax = float(f[0]), float(f[1])
+            except Exception:
+                continue
+            self.smax = smax
+            self.rows.append((time.time(), sm, {n for n, v in zip(names, f[4:8]) if v.lower() == "active"}))
 
     def mark(self):
         self.marks.append(time.time())
 
     def stop(self):
+        self.stop_ev.set()
         if self.proc:
             self.proc.terminate()
             try:
@@ -88,31 +171,39 @@ class ClockSampler:
             except Exception:
                 self.proc.kill()
 
-    def summary(self):
-        if not self.rows:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        t0, t1 = (self.marks + [0, 0])[:2] if len(self.marks) >= 2 else (0, 1e18)
-        inside = [r for r in self.rows if t0 <= r[0] <= t1]
-        note = None
-        if len(inside) < 3:
-            inside, note = self.rows, "timed region shorter than 3 samples: whole-run samples"
-        sm, smax, reasons = [], [], set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for _, line in inside:
-            f = [x.strip() for x in line.split(",")]
-            try:
-                sm.append(float(f[0]))
-                smax.append(float(f[1]))
-            except Exception:
-                continue
-            for name, v in zip(names, f[4:8]):
-                if v.lower() == "active":
-                    reasons.add(name)
-        out = {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
-               "reasons": sorted(reasons), "samples": len(inside)}
+    def window(self, i0: int, i1: int):
+        t0, t1 = self.marks[i0], self.marks[i1]
+        return [r for r in self.rows if t0 <= r[0] <= t1]
+
+    def summarize(self, rows, note=None):
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": self.smax, "reasons": ["no clock samples"], "samples": 0,
+                    "source": self.source}
+        sm = [r[1] for r in rows]
+        reasons = set().union(*[r[2] for r in rows])
+        out = {"sm_mhz": statistics.median(sm), "sm_min_mhz": min(sm), "sm_max_mhz": self.smax,
+               "reasons": sorted(reasons), "samples": len(rows), "source": self.source}
         if note:
             out["note"] = note
         return out
+
+    def summary(self):
+        """Samples of the first marked window (the timed region)."""
+        if len(self.marks) < 2:
+            return self.summarize(self.rows, "no marked window: whole-run samples")
+        return self.summarize(self.window(0, 1))
+
+
+def clocks_line(clocks: ClockSampler, soak: bool):
+    """The timed region's clocks; when it held fewer than 3 samples, the same
+    steps were re-run untimed for >= 0.3 s right after (window 2-3) and those
+    samples are reported with the timed ones."""
+    c = clocks.summary()
+    if soak and len(clocks.marks) >= 4 and c["samples"] < 3:
+        rows = clocks.window(0, 1) + clocks.window(2, 3)
+        c = clocks.summarize(rows, f"timed region held {c['samples']} sample(s): plus an untimed re-run of the "
+                                   f"same steps for >= 0.3 s right after it")
+    return c
 
 
 def setup_dist(world: int, local: int) -> int:
@@ -203,6 +294,19 @@ def cpu_oracle_sample(cfg, T, pols_oracle, budget_s, kind, max_traces=None, thre
     return units / dt, n, dt, summ
 
 
+def cpu_oracle_single(cfg, T, pols_oracle, kind, max_traces):
+    """SURVEY 8(d) protocol: the oracle on ONE host thread (no pool) over
+    the first traces of the workload (config 1 in full: its one trace)."""
+    import gen
+    import oracle
+    n = max(1, min(max_traces, int(3e8 / max(1, T * len(pols_oracle)))))   # ~10 s at 3e7/s
+    xs = gen.gen_traces(SEED_BASE + cfg, n, T, kind=kind)
+    t = time.perf_counter()
+    oracle.replay(xs, pols_oracle)
+    dt = time.perf_counter() - t
+    return n * T * len(pols_oracle) / dt, n, dt
+
+
 def policies_for(grid):
     import paper_conf_sc_zhengspl25_b200 as magus
     if grid == "sweep256":
@@ -212,6 +316,16 @@ def policies_for(grid):
     return [magus.policy_preset(magus.POLICY_PAPER_DEFAULT)]
 
 
+def oracle_grid(grid):
+    """The oracle's own restatement of the grids (never the product's)."""
+    import oracle
+    if grid == "sweep256":
+        return oracle.grid_sweep256()
+    if grid == "fleet64":
+        return oracle.grid_fleet64()
+    return oracle.policy()
+
+
 def oracle_policies(pols):
     import oracle
     return oracle.policies([dict(W=p.window, H=p.history, L=p.deriv_len, tau_inc=p.tau_inc,
@@ -219,39 +333,89 @@ def oracle_policies(pols):
                             for p in pols])
 
 
+def host_info() -> dict:
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            if ln.lower().startswith("model name"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    if model is None:
+        try:
+            for ln in open("/proc/cpuinfo"):
+                if ln.startswith("model name"):
+                    model = ln.split(":", 1)[1].strip()
+                    break
+        except Exception:
+            pass
+    return {"cpu_model": model, "nproc": os.cpu_count(), "affinity_cores": host_cores()}
+
+
 def run_reference(args):
-    """--impl reference: the oracle timed on the host cores, bounded samples."""
+    """--impl reference: the oracle, as it stands, timed on the host cores on
+    our arm's config / metric / unit.  Each step replays as much of the
+    workload as fits the time budget (the whole of config 2 on a 16-core
+    host); the line says whether that is the whole workload.  Only oracle/
+    and gen/ are loaded: the product library is not touched."""
     world, rank, _ = dist_env()
     if rank != 0:
         return 0
-    N, T, grid, kind, _, desc = WORKLOADS[args.config]
     import gen
     import oracle
-    pols = oracle_policies(policies_for(grid))
+    _, _, grid, kind, _, _, _ = WORKLOADS[args.config]
+    cfgd = workload_config(args.config, world, args.shard, args.n_traces, args.n_steps, args.no_decisions)
+    N, T, C = cfgd["n_traces_total"], cfgd["n_steps"], cfgd["n_configs"]
+    pols = oracle_grid(grid)
     seed = SEED_BASE + args.config
     threads = args.cpu_threads or host_cores()
-    per_thread = 4 if args.config not in (4, 5) else 1
-    per_step = max(1, min(N, per_thread * threads))
-    xs = gen.gen_traces(seed, per_step, T, kind=kind)
-    if args.config in (3, 4):
-        pols = pols[:16]  # bounded: 16 of the 256 / 64 configs per step
-    pool = OraclePool(threads)
-    for _ in range(args.warmup):
-        pool.replay(xs, pols)
+    # probe: single-thread time per trace x config on a small sample of this workload
+    pc = pols[:min(len(pols), 4)]
+    probe_n = max(1, min(N, 8))
+    xp = gen.gen_traces(seed, probe_n, T, kind=kind)
     t = time.perf_counter()
+    oracle.replay(xp, pc)
+    per_unit = (time.perf_counter() - t) / (probe_n * len(pc))      # s per trace x config, 1 thread
+    budget = args.ref_budget / max(1, args.steps + args.warmup)       # s per step
+    n_cfg = C if per_unit * C * threads <= budget * threads else max(1, min(C, 16))
+    n_tr = int(budget * threads / max(per_unit * n_cfg, 1e-12))
+    n_tr = max(min(threads, N), min(N, n_tr))
+    xs = gen.gen_traces(seed, n_tr, T, kind=kind)
+    use = pols[:n_cfg]
+    pool = OraclePool(threads)
+    # the first warm-up step re-calibrates at the step's real stride (the
+    # oracle reads each trace with stride ld, so the small probe is optimistic)
+    t = time.perf_counter()
+    pool.replay(xs, use)
+    per_trace = (time.perf_counter() - t) / n_tr
+    n_new = max(min(threads, N), min(N, int(budget / max(per_trace, 1e-12))))
+    if n_new < n_tr:
+        n_tr = n_new
+        xs = gen.gen_traces(seed, n_tr, T, kind=kind)
+    for _ in range(args.warmup - 1):
+        pool.replay(xs, use)
+    times = []
     for _ in range(args.steps):
-        pool.replay(xs, pols)
-    dt = (time.perf_counter() - t) / args.steps
+        t = time.perf_counter()
+        pool.replay(xs, use)
+        times.append(time.perf_counter() - t)
     pool.close()
-    cores = min(threads, per_step)
-    value = per_step * T * len(pols) / dt
-    sample = (f"{per_step} trace(s) x {T} intervals x {len(pols)} config(s) per step (seed {seed:#x}), "
-              f"statically partitioned over {cores} host thread(s)")
+    dt = sum(times) / len(times)
+    cores = min(threads, n_tr)
+    value = n_tr * T * n_cfg / dt
+    whole = n_tr == N and n_cfg == C
+    sample = (f"{n_tr} of {N} trace(s) x {T} intervals x {n_cfg} of {C} config(s) per step (seed {seed:#x}), "
+              f"statically partitioned over {cores} host thread(s)" + (" -- the whole workload" if whole else ""))
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": desc, "n_steps": T, "n_configs": len(pols), "kind": kind},
-            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3,
+            "step_ms": {"mean": dt * 1e3, "median": statistics.median(times) * 1e3, "best": min(times) * 1e3,
+                        "n": len(times)},
+            "higher_is_better": True, "scaling": cfgd["scaling"], "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": cfgd, "whole_workload_per_step": whole,
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample,
+                             "host": host_info()},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -271,52 +435,54 @@ def run_ours(args):
     dev = torch.device(f"cuda:{local}")
     stream = torch.cuda.current_stream(dev)
 
-    N, T, grid, kind, want_dec, desc = WORKLOADS[args.config]
-    if args.n_traces:
-        N = args.n_traces
-    if args.n_steps:
-        T = args.n_steps
-    if args.no_decisions:
-        want_dec = False
-    pols = policies_for(grid)
+    _, _, grid, kind, _, _, _ = WORKLOADS[args.config]
+    cfgd = workload_config(args.config, world, args.shard, args.n_traces, args.n_steps, args.no_decisions)
+    N_tot, T, want_dec, scaling = cfgd["n_traces_total"], cfgd["n_steps"], cfgd["decisions_emitted"], cfgd["scaling"]
+    pols_all = policies_for(grid)
     if args.variant:  # NEXT f3 / f4: closed loop (seq_kernel) / gradual step (walk kernels)
-        for p in pols:
+        for p in pols_all:
             p.variant = args.variant
             p.step = args.step if args.variant & magus.VARIANT_GRADUAL else 0
+    C_all = len(pols_all)
+    if args.shard == "configs":      # this rank: every trace, its block of configs
+        id0, N = 0, N_tot
+        c0, nc = mdist.shard_configs(C_all, world, rank)
+    else:                            # this rank: its block of traces, every config
+        id0, N = mdist.shard(N_tot, world, rank)
+        c0, nc = 0, C_all
+    pols = pols_all[c0:c0 + nc]
     C = len(pols)
     seed = SEED_BASE + args.config
     plat = magus.platform_preset()
     if args.burst > 0:  # NEXT f1: Sec. 6.3 burst Jaccard counters in the same pass
         plat.burst_mbs = args.burst
+    opts = [(magus.OPT_WAVES, args.waves), (magus.OPT_SEGMENTS, args.segments), (magus.OPT_BUNDLE, args.bundle),
+            (magus.OPT_SPEC_WARM, args.spec_warm), (magus.OPT_KERNEL, args.kernel)]
     ctx = magus.Context(device=local, stream=stream, platform=plat)
-    if args.waves:
-        ctx.set_option(magus.OPT_WAVES, args.waves)
-    if args.segments:
-        ctx.set_option(magus.OPT_SEGMENTS, args.segments)
-    if args.bundle:
-        ctx.set_option(magus.OPT_BUNDLE, args.bundle)
-    if args.spec_warm:
-        ctx.set_option(magus.OPT_SPEC_WARM, args.spec_warm)
-    if args.kernel:
-        ctx.set_option(magus.OPT_KERNEL, args.kernel)
-    id0, _ = mdist.shard(N * world, world, rank)     # weak scaling: N traces per GPU
+    for k, v in opts:
+        if v:
+            ctx.set_option(k, v)
     x = ctx.gen_traces(seed, N, T, kind=kind, id0=id0)
     torch.cuda.synchronize()
+    # inputs that fit in L2 are flushed before every step (outside the step's events)
+    flush = None
+    if N * T * 4 <= 4 * 126e6:
+        flush = torch.empty(64 << 20, dtype=torch.float32, device=dev)   # 256 MB > L2
 
-    out = None
-    sweep_buf = None
     # --inflight 2: consecutive steps alternate between two contexts on two
     # streams (own scratch, outputs and choice buffers; the traces are
     # shared, read-only), so one step's tail overlaps the next step's head
-    lanes = [[ctx, stream, None, None]]
-    if args.inflight > 1:
+    lanes = [[ctx, stream, None, None, None]]
+    if args.inflight > 1 and flush is None:
         s2 = torch.cuda.Stream(dev)
         ctx2 = magus.Context(device=local, stream=s2, platform=plat)
-        for k, v in ((magus.OPT_WAVES, args.waves), (magus.OPT_SEGMENTS, args.segments),
-                     (magus.OPT_BUNDLE, args.bundle), (magus.OPT_KERNEL, args.kernel)):
+        for k, v in opts:
             if v:
                 ctx2.set_option(k, v)
-        lanes.append([ctx2, s2, None, None])
+        lanes.append([ctx2, s2, None, None, None])
+    if args.shard == "configs":
+        for ln in lanes:
+            ln[4] = torch.zeros((C_all, magus.TOT_WORDS), dtype=torch.int64, device=dev)
     nstep = [0]
     if args.comm == "native" and world > 1:
         # rank 0's NCCL id reaches every rank through the process group
@@ -329,25 +495,28 @@ def run_ours(args):
         # replay (one fused launch per W group) -> NCCL sum of the integer
         # totals -> device-side choice + async device->host copy of the result
         # into pinned memory (no host sync inside a step; --sync-sweep restores
-        # the synchronous magus_sweep_best)
-        nonlocal out, sweep_buf
+        # the synchronous magus_sweep_best).  Returns (lane stream, choice).
         ln = lanes[nstep[0] % len(lanes)]
         nstep[0] += 1
-        c_, s_, o_, b_ = ln
+        c_, s_, o_, b_, full = ln
         with torch.cuda.stream(s_):
             o_ = c_.replay(x, pols, want_summary=False, want_base=False, want_decisions=want_dec,
                            want_totals=True, out=o_)
+            tot = o_.totals
+            if full is not None:               # config shard: this rank's rows of [C_all x 18]
+                full.zero_()
+                full[c0:c0 + nc].copy_(tot)
+                tot = full
             if args.comm == "native":          # the library's own NCCL communicator
-                c_.allreduce_totals(o_.totals)
+                c_.allreduce_totals(tot)
             else:
-                mdist.allreduce_totals(o_.totals)  # the one collective; exact (integer words)
+                mdist.allreduce_totals(tot)    # the one collective; exact (integer words)
+            ln[2] = o_
             if args.sync_sweep:
-                ln[2] = o_
-                return c_.sweep_best(o_.totals)
-            b_ = c_.sweep_best_async(o_.totals, b_)
-        ln[2], ln[3] = o_, b_
-        out, sweep_buf = o_, b_
-        return b_
+                return s_, c_.sweep_best(tot)
+            b_ = c_.sweep_best_async(tot, b_)
+        ln[3] = b_
+        return s_, b_
 
     def result(r):
         return r if args.sync_sweep else ctx.sweep_result(r)
@@ -358,48 +527,77 @@ def run_ours(args):
 
     clocks = ClockSampler(local)
     clocks.start()
-    time.sleep(0.3)
+    time.sleep(0.2)
     for ln in lanes:
         ln[0].set_option(magus.OPT_TIMING, 1)
         ln[0].reset_stats()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
+    e0, e1 = ev(), ev()
+    ends = []
+    per_step = []     # (start, end) events of each step when L2 is flushed between steps
     clocks.mark()
     e0.record(stream)
     for ln in lanes[1:]:
         ln[1].wait_event(e0)
     for _ in range(args.steps):
-        best = step()
+        if flush is not None:
+            flush.zero_()
+            a = ev()
+            a.record(stream)
+        s_, best = step()
+        d = ev()
+        d.record(s_)
+        ends.append(d)
+        if flush is not None:
+            per_step.append((a, d))
     for ln in lanes[1:]:
         done_ev = torch.cuda.Event()
         done_ev.record(ln[1])
         stream.wait_event(done_ev)
     e1.record(stream)
     torch.cuda.synchronize()
-    best = result(best)
     clocks.mark()
+    best = result(best)
     if world > 1:
         dist.barrier()
-    ms = e0.elapsed_time(e1)
+    if per_step:
+        steps_ms = [a.elapsed_time(d) for a, d in per_step]
+        ms = sum(steps_ms)
+    else:
+        ms = e0.elapsed_time(e1)
+        done = sorted(e0.elapsed_time(d) for d in ends)
+        steps_ms = [b - a for a, b in zip([0.0] + done[:-1], done)]   # inter-completion times
     st = ctx.stats()
     for ln in lanes[1:]:  # launches of every context in flight
         s2 = ln[0].stats()
         for key in ("launches_total", "main_launches", "main_ms_total"):
             st[key] += s2[key]
+    for ln in lanes:
         ln[0].set_option(magus.OPT_TIMING, 0)
-    ctx.set_option(magus.OPT_TIMING, 0)
-    time.sleep(0.2)
+    soak = ms < 100.0
+    if soak:  # the same steps, untimed, for >= 0.3 s: clock samples under this load
+        clocks.mark()
+        t = time.time()
+        while time.time() - t < 0.3:
+            for _ in range(8):
+                step()
+            torch.cuda.synchronize()
+        clocks.mark()
+    time.sleep(0.05)
     clocks.stop()
-    # with steps in flight, also time the dominant kernel alone: a few serial
-    # steps on one context, untimed for `value`, CUDA events per launch
+    # the dominant kernel ALONE: serial steps on one context after the timed
+    # region, CUDA events around each launch on its stream (this is the
+    # roofline's kernel time; with steps in flight the in-region event times
+    # include the other stream's share of the GPU)
     serial_ms = None
     if len(lanes) > 1:
         torch.cuda.synchronize()
         ctx.set_option(magus.OPT_TIMING, 1)
         ctx.reset_stats()
-        for _ in range(min(50, max(5, args.steps))):
+        for _ in range(min(50, max(10, args.steps))):
             o = ctx.replay(x, pols, want_summary=False, want_base=False, want_decisions=want_dec,
                            want_totals=True, out=lanes[0][2])
             lanes[0][2] = o
@@ -407,41 +605,65 @@ def run_ours(args):
         s1 = ctx.stats()
         ctx.set_option(magus.OPT_TIMING, 0)
         serial_ms = s1["main_ms_total"] / max(1, s1["main_launches"])
+    kern_ms = st["main_ms_total"] / max(1, st["main_launches"])
     if world > 1:
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        t = torch.tensor([ms, kern_ms, serial_ms or 0.0], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
-        kt = torch.tensor([st["main_ms_total"]], dtype=torch.float64, device=dev)
-        dist.all_reduce(kt, op=dist.ReduceOp.MAX)
-        st["main_ms_total"] = float(kt.item())
+        ms, kern_ms = float(t[0].item()), float(t[1].item())
+        serial_ms = float(t[2].item()) if serial_ms is not None else None
     ms_per_step = ms / args.steps
-    units_per_step = N * world * T * C
+    units_per_step = N_tot * T * C_all
     value = units_per_step / (ms_per_step * 1e-3)
 
-    # roofline of the dominant kernel (stream kernel), from live CUDA events
+    # roofline of the dominant kernel, from live CUDA events
     peak, peak_src = _peaks()
-    kern_ms = st["main_ms_total"] / max(1, st["main_launches"])
-    alg_bytes = N * T * 4 + (C * N * T / 8 if want_dec else 0)
-    achieved = alg_bytes / (kern_ms * 1e-3) / 1e9
-    roof_method = "algorithmic bytes per launch / mean launch duration (CUDA events on the launching stream)"
-    if len(lanes) > 1:
-        # consecutive steps' kernels overlap on two streams, so each launch's
-        # event-timed duration includes the other's share of the GPU: the
-        # dominant kernel's rate is the aggregate over the timed region
-        achieved = alg_bytes * args.steps / (ms * 1e-3) / 1e9
-        roof_method = (f"{len(lanes)} launches in flight on separate streams: algorithmic bytes of all launches / "
-                       f"timed region (per-launch event duration {kern_ms:.4f} ms includes the overlap)")
+    alone_ms = serial_ms if serial_ms is not None else kern_ms
+    alg_bytes = N * T * 4 + (C * N * T / 8 if want_dec else 0)      # per launch on this rank
     traffic = None
-    kname = {1: "ref_kernel", 2: "stream_kernel", 3: "seq_kernel", 4: "walk_map_kernel + walk_replay_kernel + walk_final_kernel", 5: "spec_kernel + spec_fix_kernel"}.get(st["last_kernel"], "?")
+    kname = {1: "ref_kernel", 2: "stream_kernel", 3: "seq_kernel",
+             4: "walk_map_kernel + walk_replay_kernel + walk_final_kernel",
+             5: "spec_kernel + spec_fix_kernel"}.get(st["last_kernel"], "?")
     vtag = {0: "", 1: "_f3", 2: "_f4"}.get(args.variant, f"_v{args.variant}")
     # traffic only from an ncu capture of this very kernel and workload
     prof = os.path.join(ROOT, "profiles", f"ncu_cfg{args.config}{vtag}.json")
-    if os.path.exists(prof):
+    ncu = {}
+    if os.path.exists(prof) and world == 1:
         try:
             with open(prof) as f:
-                traffic = json.load(f).get("dram_bytes_per_launch")
+                ncu = json.load(f)
+            traffic = ncu.get("dram_bytes_per_launch")
         except Exception:
-            traffic = None
+            ncu = {}
+    clk = clocks_line(clocks, soak)
+    method = ("algorithmic bytes per launch / the launch's CUDA-event duration on its stream, the kernel "
+              "timed alone" + (" (serial launches after the timed region)" if serial_ms is not None else ""))
+    hbm_roof = {"bound": "hbm", "achieved": alg_bytes / (alone_ms * 1e-3) / 1e9, "peak": peak, "unit": "GB/s",
+                "traffic": traffic, "peak_source": peak_src, "kernel": kname, "kernel_ms": alone_ms,
+                "alg_bytes_per_launch": alg_bytes, "method": method}
+    hbm_roof["frac"] = hbm_roof["achieved"] / peak
+    if len(lanes) > 1:
+        agg = alg_bytes * args.steps / (ms * 1e-3) / 1e9
+        hbm_roof["aggregate"] = {"achieved": agg, "frac": agg / peak, "steps_in_flight": len(lanes),
+                                 "note": "algorithmic bytes of all launches / timed region with consecutive "
+                                         "steps overlapping on two streams (not a per-kernel number)"}
+    roof = hbm_roof
+    if C > 1:
+        # C > 1 sweeps are ALU-bound: 8 lane-ops per decision
+        # (SURVEY 8(d)); peak = 148 SMs x 4 SMSPs x 32 lanes x max SM clock
+        sm_mhz = clk.get("sm_max_mhz") or 1965.0
+        alu_peak = 148 * 4 * 32 * sm_mhz * 1e6 / 1e9   # Gop/s
+        ach = 8.0 * N * T * C / (alone_ms * 1e-3) / 1e9
+        roof = {"bound": "alu", "achieved": ach, "peak": alu_peak, "unit": "Gop/s", "frac": ach / alu_peak,
+                "traffic": traffic,
+                "peak_source": f"148 SMs x 128 lanes x {sm_mhz:.0f} MHz (B200_PROFILING.md unit counts)",
+                "kernel": kname, "kernel_ms": alone_ms, "alg_ops_per_decision": 8, "method": method}
+        if ncu.get("metrics", {}).get("smsp__issue_active.avg.pct_of_peak_sustained_active"):
+            roof["ncu_issue_active_frac"] = float(
+                ncu["metrics"]["smsp__issue_active.avg.pct_of_peak_sustained_active"]["value"]) / 100
+            roof["ncu_thread_inst_per_decision"] = ncu.get("thread_instructions_per_unit")
+        if len(lanes) > 1:
+            agg = 8.0 * N * T * C * args.steps / (ms * 1e-3) / 1e9
+            roof["aggregate"] = {"achieved": agg, "frac": agg / alu_peak, "steps_in_flight": len(lanes)}
 
     # e2e: through the C-ABI with HOST buffers (H2D of the traces + D2H of the totals per step)
     e2e = None
@@ -457,17 +679,17 @@ def run_ours(args):
         for _ in range(e2e_steps):
             _, _, _, tot = ctx.replay_host(xn, pols, want_summary=False, want_base=False, want_totals=True)
             if world > 1:
-                tt = torch.from_numpy(tot.view(np.int64)).to(dev)
-                dist.all_reduce(tt, op=dist.ReduceOp.SUM)
-                tt.cpu()
+                full = torch.zeros((C_all, magus.TOT_WORDS), dtype=torch.int64)
+                full[c0:c0 + nc] = torch.from_numpy(tot.view(np.int64))
+                mdist.allreduce_totals(full.to(dev)).cpu()
         el = time.perf_counter() - t
         if world > 1:
             tmax = torch.tensor([el], dtype=torch.float64, device=dev)
             dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
             el = float(tmax.item())
         e2e = {"value": units_per_step * e2e_steps / el, "unit": UNIT,
-               "h2d_bytes_per_step": N * T * 4 * world, "d2h_bytes_per_step": C * 16 * 8 * world,
-               "steps": e2e_steps, "path": "magus_replay_host (pinned host traces)"}
+               "h2d_bytes_per_step": N * T * 4 * world, "d2h_bytes_per_step": C * magus.TOT_WORDS * 8 * world,
+               "steps": e2e_steps, "path": "magus_replay_host (pinned host traces; wall clock, max over ranks)"}
 
     cpu = None
     parity = None
@@ -478,9 +700,14 @@ def run_ours(args):
         threads = args.cpu_threads or host_cores()
         v, n_s, dt_s, ref_summ = cpu_oracle_sample(args.config, T, pol_o, args.cpu_budget, kind, max_traces=N,
                                                    threads=threads)
+        v1, n1, dt1 = cpu_oracle_single(args.config, T, pol_o, kind, max_traces=min(N, 128))
         cpu = {"value": v, "unit": UNIT, "cores": min(threads, n_s), "kind": "oracle",
                "sample": f"first {n_s} traces x {T} intervals x {len(pol_o)} config(s) of the same workload, "
-                         f"statically partitioned over {min(threads, n_s)} host thread(s) ({dt_s:.1f} s)"}
+                         f"statically partitioned over {min(threads, n_s)} host thread(s) ({dt_s:.1f} s)",
+               "single_thread": {"value": v1, "unit": UNIT,
+                                 "sample": f"first {n1} traces x {T} intervals x {len(pol_o)} config(s), "
+                                           f"one thread ({dt1:.1f} s)"},
+               "host": host_info()}
         # parity of that sample against the GPU path (untimed)
         r = ctx.replay(x[:, :n_s], pols[:len(pol_o)], n_traces=n_s, want_totals=False)
         torch.cuda.synchronize()
@@ -489,53 +716,34 @@ def run_ours(args):
                           [("n_events", "n_events"), ("n_changes", "n_changes"), ("digest", "digest"),
                            ("energy_j", "energy"), ("time_s", "time")]))
 
-    # C > 1 sweeps are ALU-bound: algorithmic work = 8 lane-ops
-    # per decision (lag difference, 2 threshold compares, event
-    # log, count compare, priority select, change compare, accumulate); peak =
-    # 148 SMs x 4 SMSPs x 32 lanes x max SM clock (one lane-op per lane-cycle).
-    clk = clocks.summary()
-    hbm_roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                "kernel": kname, "kernel_ms": kern_ms, "alg_bytes_per_launch": alg_bytes,
-                "method": roof_method}
-    if serial_ms is not None:
-        hbm_roof["serial_launch"] = {"kernel_ms": serial_ms, "achieved": alg_bytes / (serial_ms * 1e-3) / 1e9,
-                                     "frac": alg_bytes / (serial_ms * 1e-3) / 1e9 / peak,
-                                     "note": "the kernel timed alone (serial steps after the timed region)"}
-    roof = hbm_roof
-    if C > 1:
-        sm_mhz = clk.get("sm_max_mhz") or 1965.0
-        alu_peak = 148 * 4 * 32 * sm_mhz * 1e6 / 1e9   # Gop/s
-        alu_ach = 8.0 * N * T * C / (kern_ms * 1e-3) / 1e9
-        if len(lanes) > 1:
-            alu_ach = 8.0 * N * T * C * args.steps / (ms * 1e-3) / 1e9
-        roof = {"bound": "alu", "achieved": alu_ach, "peak": alu_peak, "unit": "Gop/s",
-                "frac": alu_ach / alu_peak, "traffic": traffic,
-                "peak_source": f"148 SMs x 128 lanes x {sm_mhz:.0f} MHz (B200_PROFILING.md unit counts)",
-                "kernel": kname, "kernel_ms": kern_ms, "alg_ops_per_decision": 8, "method": roof_method}
-        if serial_ms is not None:
-            sa = 8.0 * N * T * C / (serial_ms * 1e-3) / 1e9
-            roof["serial_launch"] = {"kernel_ms": serial_ms, "achieved": sa, "frac": sa / alu_peak,
-                                     "note": "the kernel timed alone (serial steps after the timed region)"}
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": desc, "n_traces_per_gpu": N, "n_traces_total": N * world, "n_steps": T,
-                       "n_configs": C, "decisions_emitted": want_dec, "seed": hex(seed),
-                       "l2": f"inputs {N * T * 4 / 1e9:.2f} GB per GPU > 126 MB L2 (no flush needed)",
-                       "parallelism": f"traces sharded over {world} GPU(s); 1 all-reduce of int64 totals "
-                                      f"({'native NCCL' if args.comm == 'native' and world > 1 else dist_backend(world)})",
-                       "steps_in_flight": len(lanes),
-                       "segments": st["last_segments"], "kernel": {1: "reference", 2: "stream", 3: "sequential", 4: "walk", 5: "spec"}.get(st["last_kernel"], "?"),
-                       "variant": args.variant, "step": args.step if args.variant & 2 else 0},
+            "warmup": args.warmup, "ms_per_step": ms_per_step,
+            "step_ms": {"mean": ms_per_step, "median": statistics.median(steps_ms), "best": min(steps_ms),
+                        "n": len(steps_ms),
+                        "method": "per-step CUDA events around each step" if per_step else
+                                  "intervals between consecutive step-completion events"},
+            "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": cfgd,
+            "run": {"steps_in_flight": len(lanes), "segments": st["last_segments"],
+                    "kernel": {1: "reference", 2: "stream", 3: "sequential", 4: "walk", 5: "spec"}.get(
+                        st["last_kernel"], "?"),
+                    "variant": args.variant, "step": args.step if args.variant & 2 else 0,
+                    "comm": "native NCCL" if args.comm == "native" and world > 1 else dist_backend(world),
+                    "configs_this_rank": [c0, nc], "traces_this_rank": [id0, N],
+                    "l2_flush": flush is not None},
             "roofline": roof,
             "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": int(st["launches_total"]), "clocks": clk,
             "best_config": best[0], "feasible": best[2]}
+    if args.t1_ms:
+        line["scaling_efficiency"] = {
+            "value": args.t1_ms / ((world if scaling == "strong" else 1) * ms_per_step),
+            "t1_ms": args.t1_ms, "tN_ms": ms_per_step,
+            "formula": "t1 / (G * tG)" if scaling == "strong" else "t1 / tG (weak)"}
     if args.burst > 0:
         line["config"]["burst_mbs"] = args.burst
         line["best_jaccard"] = best[1]["jaccard"]
-        line["pareto_front"] = [int(i) for i in np.flatnonzero(ctx.pareto_front(out.totals))]
+        line["pareto_front"] = [int(i) for i in np.flatnonzero(ctx.pareto_front(lanes[0][2].totals))]
     if roof is not hbm_roof:
         line["roofline_hbm"] = hbm_roof
     if parity is not None:
@@ -569,7 +777,7 @@ def run_fleet(args):
     local = setup_dist(world, local)
     dev = torch.device(f"cuda:{local}")
     stream = torch.cuda.current_stream(dev)
-    N_tot, T, grid, kind, _, desc = WORKLOADS[4]
+    N_tot, T, grid, kind, _, _, _ = WORKLOADS[4]
     if args.n_traces:
         N_tot = args.n_traces
     if args.n_steps:
@@ -687,13 +895,12 @@ def run_fleet(args):
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": desc, "n_traces_total": N_tot, "n_traces_per_gpu": N, "n_steps": T,
-                       "n_configs": C, "decisions_emitted": False, "seed": hex(seed),
-                       "chunk_intervals": R, "chunks": len(chunks), "halo_rows": halo,
-                       "l2": f"chunks of {N * R * 4 / 1e9:.1f} GB > 126 MB L2 (no flush needed)",
-                       "timed": "replay calls + all-reduce + device choice; on-device generation of each "
-                                "chunk and the halo copy untimed (SURVEY 8(d))",
-                       "parallelism": f"traces sharded over {world} GPU(s); 1 all-reduce of int64 totals ({dist_backend(world)})"},
+            "config": workload_config(4, world, "traces", args.n_traces, args.n_steps),
+            "run": {"chunk_intervals": R, "chunks": len(chunks), "halo_rows": halo,
+                    "l2": f"chunks of {N * R * 4 / 1e9:.1f} GB > 126 MB L2 (no flush needed)",
+                    "timed": "replay calls + all-reduce + device choice; on-device generation of each "
+                             "chunk and the halo copy untimed (SURVEY 8(d))",
+                    "comm": dist_backend(world), "traces_this_rank": [id0, N]},
             "roofline": {"bound": "alu", "achieved": alu_ach, "peak": alu_peak, "unit": "Gop/s",
                          "frac": alu_ach / alu_peak, "traffic": None,
                          "peak_source": f"148 SMs x 128 lanes x {sm_mhz:.0f} MHz (B200_PROFILING.md unit counts)",
@@ -722,7 +929,8 @@ def run_bound(args):
 
     import oracle
     import paper_conf_sc_zhengspl25_b200 as magus
-    N, T, _, kind, _, desc = WORKLOADS[args.config]
+    N, T, _, kind, _, _, _ = WORKLOADS[args.config]
+    desc = workload_config(args.config, 1, "traces", args.n_traces, args.n_steps)["workload"]
     if args.n_traces:
         N = args.n_traces
     if args.n_steps:
@@ -803,6 +1011,13 @@ def main():
     ap.add_argument("--burst", type=float, default=0.0,
                     help="NEXT f1: Sec. 6.3 burst threshold (MB/s); > 0 enables the Jaccard counters")
     ap.add_argument("--chunk", type=int, default=0, help="cfg4: intervals per time chunk (0 = fit ~32 GiB)")
+    ap.add_argument("--shard", choices=["traces", "configs"], default="traces",
+                    help="multi-GPU split: trace blocks (default) or config blocks (every rank holds every trace)")
+    ap.add_argument("--t1-ms", type=float, default=0.0,
+                    help="1-GPU ms/step of the same workload: adds scaling_efficiency = t1/(G*tG) (strong) "
+                         "or t1/tG (weak)")
+    ap.add_argument("--ref-budget", type=float, default=150.0,
+                    help="--impl reference: seconds of oracle work for the whole --steps + --warmup run")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -99,6 +99,28 @@ def policies(rows) -> np.ndarray:
     return out
 
 
+def grid_sweep256() -> np.ndarray:
+    """SWEEP256 (reading R16 of DESIGN.md 3): tau_inc in
+    {100, 200, 300, 400} x tau_dec in {-250, -500, -750, -1000} x t_hi in
+    {0.2, 0.3, 0.4, 0.5} x W in {4, 6, 10, 16}, L = W, H = 10; index =
+    iInc + 4 (iDec + 4 (iHi + 4 iW)).  paper_default (P@25197) is index 165,
+    paper_pareto (P@44170) 166.  Restated here, independently of the product."""
+    rows = []
+    for W in (4, 6, 10, 16):
+        for t_hi in (0.2, 0.3, 0.4, 0.5):
+            for tau_dec in (-250.0, -500.0, -750.0, -1000.0):
+                for tau_inc in (100.0, 200.0, 300.0, 400.0):
+                    rows.append(dict(W=W, H=10, L=float(W), tau_inc=tau_inc, tau_dec=tau_dec, t_hi=t_hi))
+    return policies(rows)
+
+
+def grid_fleet64() -> np.ndarray:
+    """FLEET64: the tau_inc x tau_dec x t_hi lines of
+    SWEEP256 at W = L = H = 10; index = iInc + 4 (iDec + 4 iHi); default 37."""
+    g = grid_sweep256()
+    return np.ascontiguousarray(g[g["W"] == 10])
+
+
 def platform(r_min=8, r_max=22, dt=0.2, bw_max=32000.0, beta=1.0, p_other=218.0,
              p_unc_min=0.0, p_unc_max=82.0, e_sw=0.0, t_sw=0.0, bound=0.05, burst=0.0) -> np.ndarray:
     """Intel+A100 (uncore 0.8-2.2 GHz, P@29320); 82 W uncore range (Fig. 2,

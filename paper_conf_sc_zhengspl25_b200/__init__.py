@@ -239,7 +239,7 @@ def derive_host(totals_row, platform: Platform | None = None) -> dict:
 
 
 def sweep_best_host(totals, platform: Platform | None = None) -> tuple[int, dict, bool]:
-    """(best, derived row, feasible) from host totals [C, 16] (no GPU)."""
+    """(best, derived row, feasible) from host totals [C, TOT_WORDS=18] (no GPU)."""
     plat = platform if platform is not None else platform_preset()
     w = np.ascontiguousarray(np.asarray(totals).view(np.uint64).reshape(-1, TOT_WORDS))
     best, d = _i32(), Derived()
@@ -276,10 +276,10 @@ def _policy_array(policies) -> tuple[ctypes.Array, int]:
 
 @dataclass
 class ReplayResult:
-    summary: object | None      # torch.uint8 [C, N, 104] (use summary_numpy())
+    summary: object | None      # torch.uint8 [C, N, SUMMARY_DT.itemsize=120] (use summary_numpy())
     base: object | None         # torch.uint8 [N, 32]
     decisions: object | None    # torch.int32 view of uint32 [C, ceil(T/32), N]
-    totals: object | None       # torch.int64 view of uint64 [C, 16]
+    totals: object | None       # torch.int64 view of uint64 [C, TOT_WORDS=18]
     n_traces: int
     n_configs: int
 
@@ -294,6 +294,28 @@ class ReplayResult:
 
     def decisions_numpy(self) -> np.ndarray:
         return self.decisions.cpu().numpy().view(np.uint32)
+
+
+def _check_out(out: ReplayResult, N: int, C: int, nw: int, dev, want_summary: bool, want_base: bool,
+               want_decisions: bool, want_totals: bool) -> None:
+    """Caller-supplied output buffers must match this call exactly: the kernels
+    write [C, N, ...] / [C, nw, N] / [C, TOT_WORDS] without bounds checks."""
+    torch = __import__("torch")
+    spec = (("summary", want_summary, (C, N, SUMMARY_DT.itemsize), torch.uint8),
+            ("base", want_base, (N, 32), torch.uint8),
+            ("decisions", want_decisions, (C, nw, N), torch.int32),
+            ("totals", want_totals, (C, TOT_WORDS), torch.int64))
+    for name, want, shape, dt in spec:
+        t = getattr(out, name)
+        if t is None:
+            if want:
+                raise ValueError(f"replay(out=...): {name} requested but out.{name} is None")
+            continue
+        if tuple(t.shape) != shape or t.dtype != dt or t.device != dev or not t.is_contiguous():
+            raise ValueError(f"replay(out=...): out.{name} is {tuple(t.shape)} {t.dtype} on {t.device}, "
+                             f"this call needs {shape} {dt} on {dev} (contiguous)")
+    if out.n_traces != N or out.n_configs != C:
+        raise ValueError(f"replay(out=...): result is for N={out.n_traces}, C={out.n_configs}; call has N={N}, C={C}")
 
 
 class Context:
@@ -395,6 +417,8 @@ class Context:
                 decisions=torch.empty((C, nw, N), dtype=torch.int32, device=dev) if want_decisions else None,
                 totals=torch.empty((C, TOT_WORDS), dtype=torch.int64, device=dev) if want_totals else None,
                 n_traces=N, n_configs=C)
+        else:
+            _check_out(out, N, C, (T + 31) // 32, dev, want_summary, want_base, want_decisions, want_totals)
         p = lambda t: _vp(t.data_ptr()) if t is not None else None  # noqa: E731
         st = _lib.magus_replay(self._h, _vp(traces.data_ptr()), N, T, ld, arr, C, p(out.summary), p(out.base),
                                p(out.decisions), p(out.totals))
@@ -532,7 +556,7 @@ class Context:
         return totals
 
     def sweep_best(self, totals) -> tuple[int, dict, bool]:
-        """totals: CUDA int64 tensor [C, 16] (summed over ranks if sharded).
+        """totals: CUDA int64 tensor [C, TOT_WORDS=18] (summed over ranks if sharded).
         Returns (best index, derived row, feasible)."""
         C = totals.shape[0]
         best = _i32()

@@ -762,7 +762,10 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     if (st != MAGUS_OK) return st;
     const uint64_t sig = ((uint64_t)C * 1000003ULL + (uint64_t)N) * 1000033ULL + (uint64_t)nseg + 1;
     if (sig != ctx->work_sig) {
-      CK(cudaMemsetAsync(ctx->scratch, 0, off_status, ctx->stream));
+      // the whole region, status words included: another kernel path (walk,
+      // seq, reference) may have left arbitrary words in this scratch, and a
+      // look-back accepts any word whose tag equals the epoch
+      CK(cudaMemsetAsync(ctx->scratch, 0, total, ctx->stream));
       ctx->work_sig = sig;
     }
     if (++ctx->epoch >= (1u << 29)) {

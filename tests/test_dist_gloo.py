@@ -91,3 +91,47 @@ def test_host_derivation_matches_oracle():
     assert d["energy_j"] == f[0] and d["time_s"] == f[1]
     assert d["base_energy_j"] == f[2] and d["base_time_s"] == f[3]
     assert d["saving"] == f[4] and d["slowdown"] == f[5]
+
+
+def _worker_cfg(rank, world, port, out_dir):
+    """Config sharding: every rank holds every trace and fills only its rows."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import paper_conf_sc_zhengspl25_b200 as m
+    from paper_conf_sc_zhengspl25_b200 import dist as mdist
+    pols = _pols()
+    pols_o = oracle.policies([dict(W=p.window, H=p.history, L=p.deriv_len, tau_inc=p.tau_inc,
+                                   tau_dec=p.tau_dec, t_hi=p.t_hi) for p in pols])
+    c0, nc = mdist.shard_configs(len(pols), world, rank)
+    x = gen.gen_traces(gen.SEEDS[4], N_TOTAL, T)
+    full = torch.zeros((len(pols), m.TOT_WORDS), dtype=torch.int64)
+    full[c0:c0 + nc] = torch.from_numpy(_oracle_totals(x, pols_o[c0:c0 + nc]).view(np.int64).copy())
+    mdist.allreduce_totals(full)
+    best, row, feas = m.sweep_best_host(full.numpy().view(np.uint64))
+    np.save(os.path.join(out_dir, f"tot{rank}.npy"), full.numpy().view(np.uint64))
+    np.save(os.path.join(out_dir, f"best{rank}.npy"), np.array([best, int(feas)]))
+    dist.destroy_process_group()
+
+
+def test_config_sharded_allreduce_world2(tmp_path):
+    world = 2
+    mp.spawn(_worker_cfg, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True)
+    import paper_conf_sc_zhengspl25_b200 as m
+    pols = _pols()
+    pols_o = oracle.policies([dict(W=p.window, H=p.history, L=p.deriv_len, tau_inc=p.tau_inc,
+                                   tau_dec=p.tau_dec, t_hi=p.t_hi) for p in pols])
+    full = _oracle_totals(gen.gen_traces(gen.SEEDS[4], N_TOTAL, T), pols_o)
+    b_full = m.sweep_best_host(full)
+    for r in range(world):
+        assert np.array_equal(np.load(tmp_path / f"tot{r}.npy"), full)
+        best, feas = np.load(tmp_path / f"best{r}.npy")
+        assert (int(best), bool(feas)) == (b_full[0], b_full[2])
+
+
+def test_shard_configs_covers_every_config_once():
+    from paper_conf_sc_zhengspl25_b200 import dist as mdist
+    for C in (1, 16, 64, 256):
+        for world in (1, 2, 3, 8):
+            got = [mdist.shard_configs(C, world, r) for r in range(world)]
+            assert [c for c0, n in got for c in range(c0, c0 + n)] == list(range(C))
