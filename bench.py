@@ -730,6 +730,7 @@ def run_ours(args):
                     "variant": args.variant, "step": args.step if args.variant & 2 else 0,
                     "comm": "native NCCL" if args.comm == "native" and world > 1 else dist_backend(world),
                     "configs_this_rank": [c0, nc], "traces_this_rank": [id0, N],
+                    "ranks_per_gpu": max(1, world // max(1, torch.cuda.device_count())),
                     "l2_flush": flush is not None},
             "roofline": roof,
             "cpu_baseline": cpu, "e2e": e2e,

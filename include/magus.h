@@ -428,9 +428,15 @@ enum {
                                  many waves of CTAs                          */
   MAGUS_OPT_BUNDLE = 4,       /* configs per thread sharing Alg. 1/2 work:
                                  0 auto, or force 1, 2 or 4                  */
-  MAGUS_OPT_SPEC_WARM = 5     /* kernel 5: rounds each segment's speculation
+  MAGUS_OPT_SPEC_WARM = 5,    /* kernel 5: rounds each segment's speculation
                                  replays before it (0 = auto, min(segment,
                                  1024)); any value gives the same results   */
+  MAGUS_OPT_TRACE = 6,        /* 1: the stream kernel records a per-CTA
+                                 timeline (diagnostics; magus_get_trace)     */
+  MAGUS_OPT_NARROW = 7        /* 1: the stream kernel's one-config path uses
+                                 128-trace CTAs (4 per SM) instead of the
+                                 default 512-trace CTA per SM (A/B option;
+                                 results are identical)                      */
 };
 magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value);
 
@@ -445,6 +451,13 @@ typedef struct {
                                  and were replayed again, in the last replay
                                  (read with a device sync); else 0           */
 } magus_stats;
+/* Per-CTA timeline of the last stream-kernel replay under MAGUS_OPT_TRACE
+ * (diagnostics, not the hot path): out host uint64 [cap][8] per CTA (in
+ * blockIdx order) = {start, scan end, look-back end, end} (%globaltimer ns),
+ * SM id, time segment, trace group, 1 if this CTA finalised its group.
+ * *n_out = CTAs recorded (<= cap).  Synchronises ctx's stream.
+ * INVALID_ARG without a traced replay. */
+magus_status magus_get_trace(magus_ctx ctx, uint64_t* out, int64_t cap, int64_t* n_out);
 /* Synchronises when timing is on (reads the events). */
 magus_status magus_get_stats(magus_ctx ctx, magus_stats* out);
 magus_status magus_reset_stats(magus_ctx ctx);

@@ -24,7 +24,7 @@ OK, ERR_INVALID_ARG, ERR_NOT_INITIALIZED, ERR_CUDA, ERR_NCCL, ERR_OOM, ERR_UNSUP
 POLICY_PAPER_DEFAULT, POLICY_PAPER_PARETO = 0, 1
 PLATFORM_INTEL_A100, PLATFORM_INTEL_MAX1550 = 0, 1
 GEN_MIX, GEN_ADVERSARIAL = 0, 1
-OPT_KERNEL, OPT_SEGMENTS, OPT_TIMING, OPT_WAVES, OPT_BUNDLE, OPT_SPEC_WARM = 0, 1, 2, 3, 4, 5
+OPT_KERNEL, OPT_SEGMENTS, OPT_TIMING, OPT_WAVES, OPT_BUNDLE, OPT_SPEC_WARM, OPT_TRACE, OPT_NARROW = 0, 1, 2, 3, 4, 5, 6, 7
 KERNEL_AUTO, KERNEL_REFERENCE, KERNEL_STREAM, KERNEL_SEQUENTIAL, KERNEL_WALK, KERNEL_SPEC = 0, 1, 2, 3, 4, 5
 TOT_WORDS = 18
 TOT_NAMES = ["n_traces", "n_viol", "events", "hi_rounds", "msr_writes", "changes", "min_dec",
@@ -125,6 +125,7 @@ _lib.magus_pareto_front_host.argtypes = [ctypes.POINTER(Platform), _vp, _i32, _v
 _lib.magus_sweep_best_host.argtypes = [ctypes.POINTER(Platform), _vp, _i32, ctypes.POINTER(_i32),
                                        ctypes.POINTER(Derived)]
 _lib.magus_reset_stats.argtypes = [_vp]
+_lib.magus_get_trace.argtypes = [_vp, _vp, _i64, ctypes.POINTER(_i64)]
 _lib.magus_comm_unique_id.argtypes = [_vp]
 _lib.magus_comm_init.argtypes = [_vp, _vp, _i32, _i32]
 _lib.magus_allreduce_totals.argtypes = [_vp, _vp, _i32]
@@ -134,7 +135,7 @@ for _f in ("magus_init", "magus_destroy", "magus_set_stream", "magus_policy_pres
            "magus_get_stats", "magus_reset_stats", "magus_policy_inspect", "magus_platform_inspect", "magus_derive_host",
            "magus_sweep_best_host", "magus_pareto_front", "magus_pareto_front_host",
            "magus_replay_levels", "magus_offline_bound", "magus_sweep_best_async",
-           "magus_comm_unique_id", "magus_comm_init", "magus_allreduce_totals"):
+           "magus_comm_unique_id", "magus_comm_init", "magus_allreduce_totals", "magus_get_trace"):
     getattr(_lib, _f).restype = ctypes.c_int
 
 EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_string", "magus_last_error",
@@ -146,7 +147,7 @@ EXPORTED = ["magus_init", "magus_destroy", "magus_set_stream", "magus_status_str
             "magus_replay_levels", "magus_offline_bound", "magus_sweep_best_async",
             "magus_replay_resume", "magus_resume_state_bytes", "magus_resume_halo",
             "magus_gen_traces_resume", "magus_gen_state_bytes",
-            "magus_comm_unique_id", "magus_comm_init", "magus_allreduce_totals"]
+            "magus_comm_unique_id", "magus_comm_init", "magus_allreduce_totals", "magus_get_trace"]
 COMM_ID_BYTES = 128
 VARIANT_CLOSED_LOOP, VARIANT_GRADUAL = 1, 2
 
@@ -369,6 +370,16 @@ class Context:
 
     def reset_stats(self):
         self._check(_lib.magus_reset_stats(self._h), "reset_stats")
+
+    def trace(self) -> np.ndarray:
+        """Per-CTA timeline of the last traced stream replay (OPT_TRACE):
+        uint64 [CTAs, 8] = start, scan end, look-back end, end (ns), SM,
+        segment, trace group, finalised-the-group flag."""
+        cap = self.stats()["last_grid"]
+        out = np.zeros((max(cap, 1), 8), np.uint64)
+        n = _i64()
+        self._check(_lib.magus_get_trace(self._h, _vp(out.ctypes.data), cap, ctypes.byref(n)), "get_trace")
+        return out[:n.value]
 
     # -- the API --
     def gen_traces(self, seed: int, n_traces: int, n_steps: int, kind: int = GEN_MIX, id0: int = 0,

@@ -25,7 +25,11 @@ struct magus_ctx_s {
   std::string err;
   int sms = 148;
   // options
-  int64_t opt_kernel = 0, opt_segments = 0, opt_timing = 0, opt_waves = 0;
+  int64_t opt_kernel = 0, opt_segments = 0, opt_timing = 0, opt_waves = 0, opt_trace = 0, opt_narrow = 0;
+  void* trace_dev = nullptr;   // MAGUS_OPT_TRACE timeline [trace_cap][8]
+  int64_t trace_cap = 0, trace_n = 0;
+  bool trace_armed = false;          // scratch holds a timeline address
+  void* trace_slot_host[2] = {nullptr, nullptr};  // [0] the address, [1] NULL
   // device scratch
   void* scratch = nullptr;
   size_t scratch_bytes = 0;
@@ -210,12 +214,18 @@ const int32_t* dev_cidx(magus_ctx ctx, int64_t off) {
 }
 
 int ctas_per_sm(magus_ctx ctx, int W, int H, int NB) {
-  auto key = std::make_pair(W * 8 + NB, H);
+  const bool burst = ctx->dplat.burst_on != 0, narrow = ctx->opt_narrow != 0;
+  auto key = std::make_pair((W * 8 + NB) * 4 + (burst ? 2 : 0) + (narrow ? 1 : 0), H);
   auto it = ctx->ctas_cache.find(key);
   if (it != ctx->ctas_cache.end()) return it->second;
-  int v = stream_ctas_per_sm(W, H, NB);
+  int v = stream_ctas_per_sm(W, H, NB, burst, narrow);
   ctx->ctas_cache[key] = v;
   return v;
+}
+
+int64_t stream_groups(magus_ctx ctx, int64_t N, int W, int H, int NB) {  // CTAs per (segment, bundle)
+  const int tr = stream_cta_traces(W, H, NB, ctx->dplat.burst_on != 0, ctx->opt_narrow != 0);
+  return (N + tr - 1) / tr;
 }
 
 magus_status encode_tmap(magus_ctx ctx, CUtensorMap* map, const float* x, int64_t N, int64_t T,
@@ -462,6 +472,7 @@ magus_status magus_destroy(magus_ctx ctx) {
     if (ctx->best_pinned) cudaFreeHost(ctx->best_pinned);
     if (ctx->lam_dev) cudaFree(ctx->lam_dev);
     if (ctx->mul_dev) cudaFree(ctx->mul_dev);
+    if (ctx->trace_dev) cudaFree(ctx->trace_dev);
     if (ctx->sweep_dev) cudaFree(ctx->sweep_dev);
     if (ctx->stage_dev) cudaFree(ctx->stage_dev);
     if (ctx->pol_copied) cudaEventDestroy(ctx->pol_copied);
@@ -504,6 +515,12 @@ magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value) {
       if (value != 0 && value != 1 && value != 2 && value != 4)
         return fail(ctx, MAGUS_ERR_INVALID_ARG, "bundle option must be 0, 1, 2 or 4");
       ctx->opt_bundle = value;
+      return MAGUS_OK;
+    case MAGUS_OPT_TRACE:
+      ctx->opt_trace = value ? 1 : 0;
+      return MAGUS_OK;
+    case MAGUS_OPT_NARROW:
+      ctx->opt_narrow = value ? 1 : 0;
       return MAGUS_OK;
     case MAGUS_OPT_WAVES:
       if (value < 0 || value > 64) return fail(ctx, MAGUS_ERR_INVALID_ARG, "waves not in [0, 64]");
@@ -602,7 +619,7 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
         double cost = 0.0;
         for (auto& g : ctx->groups) {
           const int64_t slots = (int64_t)ctx->sms * std::max(1, ctas_per_sm(ctx, g.W, g.H, g.NB));
-          const int64_t ctas = ngroups * g.nbund * cand;
+          const int64_t ctas = stream_groups(ctx, N, g.W, g.H, g.NB) * g.nbund * cand;
           const int64_t halo = cand > 1 ? ((g.W + g.H - 1 + 31) / 32) * 32 : 0;
           cost += (double)((ctas + slots - 1) / slots) * (double)(len + halo + 96);
         }
@@ -790,6 +807,28 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     wk.tb = (int32_t)tb;       // global interval of buffer row 0
     wk.ts = (int32_t)(tb + ts);  // first interval decided (global)
     wk.carry = nullptr;
+    ctx->trace_n = 0;
+    if (ctx->opt_trace || ctx->trace_armed) {  // the timeline address (or NULL) in scratch
+      void* tp = nullptr;
+      if (ctx->opt_trace) {
+        int64_t grid_all = 0;
+        for (auto& g : ctx->groups) grid_all += stream_groups(ctx, N, g.W, g.H, g.NB) * nseg * g.nbund;
+        if (grid_all > ctx->trace_cap) {
+          CK(cudaStreamSynchronize(ctx->stream));
+          if (ctx->trace_dev) cudaFree(ctx->trace_dev);
+          ctx->trace_dev = nullptr;
+          ctx->trace_cap = 0;
+          CK(cudaMalloc(&ctx->trace_dev, 64 * (size_t)grid_all));
+          ctx->trace_cap = grid_all;
+        }
+        tp = ctx->trace_dev;
+        ctx->trace_n = grid_all;
+      }
+      ctx->trace_slot_host[0] = tp;   // (a pageable source is staged before the call returns)
+      CK(cudaMemcpyAsync((uint32_t*)sp + kTraceSlotWords, &ctx->trace_slot_host[ctx->opt_trace ? 0 : 1],
+                         sizeof(void*), cudaMemcpyHostToDevice, ctx->stream));
+      ctx->trace_armed = ctx->opt_trace != 0;
+    }
     if (rs) {  // accumulators and carries live in the caller's state
       wk.acc = (unsigned long long*)rs->state;
       wk.carry = (uint32_t*)((char*)rs->state + 8 * (size_t)kAccFields * (size_t)(C * N));
@@ -819,7 +858,7 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
       auto& g = ctx->groups[gi];
       int grid = 0;
       int r = launch_stream(ctx->stream, &map, &map_mul, N, tb + T, dev_policies(ctx), dev_cidx(ctx, g.off), g.nbund,
-                            g.NB, g.W, g.H, ctx->dplat, nseg, seg_len, wk, &grid);
+                            g.NB, g.W, g.H, ctx->dplat, nseg, seg_len, wk, ctx->opt_narrow != 0, &grid);
       if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "stream kernel launch");
       launched += r;
       grid_total += grid;
@@ -1144,6 +1183,17 @@ magus_status magus_gen_traces_resume(magus_ctx ctx, uint64_t seed, int64_t id0, 
   if (launch_gen_resume(ctx->stream, seed, id0, N, t0, n_rows, ld, kind, state, out) < 0)
     return cuda_fail(ctx, cudaGetLastError(), "gen kernel launch");
   ctx->launches += 1;
+  return MAGUS_OK;
+}
+
+magus_status magus_get_trace(magus_ctx ctx, uint64_t* out, int64_t cap, int64_t* n_out) {
+  if (!ctx || !out || cap < 0 || !n_out) return MAGUS_ERR_INVALID_ARG;
+  if (!ctx->trace_dev || ctx->trace_n == 0) return fail(ctx, MAGUS_ERR_INVALID_ARG, "no traced replay");
+  DeviceGuard dg(ctx->device);
+  const int64_t n = std::min(cap, ctx->trace_n);
+  CK(cudaMemcpyAsync(out, ctx->trace_dev, 64 * (size_t)n, cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  *n_out = n;
   return MAGUS_OK;
 }
 

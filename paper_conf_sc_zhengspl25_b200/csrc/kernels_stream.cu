@@ -41,12 +41,21 @@
 namespace magus {
 namespace {
 
-constexpr int kTraces = 128;
+constexpr int kBox = 128;   // traces per TMA box ([32 steps x 128 traces], 16 KB)
 constexpr int kRows = 32;
-constexpr int kStageFloats = kTraces * kRows;           // 16 KB
-constexpr int kConsumerWarps = kTraces / 32;
-constexpr int kThreads = kTraces + 32;                  // + producer warp
-constexpr uint32_t kStageBytes = kStageFloats * 4;
+// A CTA owns TR traces (TR / 128 boxes per stage; the stage is laid out
+// box-major, [box][32 steps][128 traces]).  TR = 512 for one config per
+// thread (one CTA per SM: its 16 consumer warps share one ring, so they
+// cannot drift apart the way 4 independent CTAs on an SM did), 128 else.
+template <int TR>
+struct Cta {
+  static constexpr int traces = TR;
+  static constexpr int boxes = TR / kBox;
+  static constexpr int stage_floats = TR * kRows;            // 16 / 64 KB
+  static constexpr uint32_t stage_bytes = stage_floats * 4;
+  static constexpr int consumer_warps = TR / 32;
+  static constexpr int threads = TR + 32;                    // + producer warp
+};
 constexpr int kTotAcc = kTotAccWords;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -125,8 +134,24 @@ __device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p) {
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
-__device__ __forceinline__ void consumer_sync() {  // the 128 consumer threads only
-  asm volatile("bar.sync 1, %0;" ::"n"(kTraces) : "memory");
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// MAGUS_OPT_TRACE: slot i of this CTA's timeline row (the CTA index is
+// re-read here so no address stays live across the scan)
+__device__ __forceinline__ unsigned long long* trace_buf(const StreamWork& wk) {
+  return *reinterpret_cast<unsigned long long* volatile*>(wk.ticket + kTraceSlotWords);
+}
+__device__ __forceinline__ void trace_put(unsigned long long* tr, int i, unsigned long long v) {
+  uint32_t cta;
+  asm volatile("mov.u32 %0, %%ctaid.x;" : "=r"(cta));
+  tr[8ull * cta + i] = v;
+}
+template <int TR>
+__device__ __forceinline__ void consumer_sync() {  // the TR consumer threads only
+  asm volatile("bar.sync 1, %0;" ::"n"(TR) : "memory");
 }
 
 // ---- Alg. 2, bit-parallel: bit i of the result = (#events at positions
@@ -233,17 +258,17 @@ __device__ __forceinline__ uint32_t tail_mask(int64_t p0, int64_t T) {
   return (p0 + 32 <= T) ? ~0u : ((1u << (uint32_t)(T - p0)) - 1u);
 }
 
-template <int W_T>
+template <int W_T, int TR>
 struct Stages {
   // register lag (compile-time W): a stage is free once its word is read;
   // runtime W reads the lag from the previous stage, held one word longer.
   static constexpr int n = W_T > 0 ? 3 : 4;
-  static constexpr int smem = n * kStageFloats * 4;
+  static constexpr int smem = n * Cta<TR>::stage_floats * 4;
 };
 // CTAs per SM the launch bounds aim for: NB configs per thread cost registers
-template <int W_T, int NB>
+template <int W_T, int NB, int TR>
 struct Occ {
-  static constexpr int v = NB == 1 ? (W_T > 0 ? 4 : 3) : 3;
+  static constexpr int v = TR > 128 ? 1 : (NB == 1 ? (W_T > 0 ? 4 : 3) : 3);
 };
 
 // Per-config state of a bundle (NB configs that share W, H, L, tau_inc and
@@ -270,14 +295,19 @@ struct BundleSmem {  // rarely touched, per (config slot, thread)
   uint32_t dwa, pre_dec_a;
 };
 
-template <int W_T, int H_T, int NB, bool BURST>
-__global__ void __launch_bounds__(kThreads, Occ<W_T, NB>::v)
+template <int W_T, int H_T, int NB, bool BURST, int TR>
+__global__ void __launch_bounds__(Cta<TR>::threads, Occ<W_T, NB, TR>::v)
 stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ CUtensorMap tmul,
               int64_t N, int64_t T,
               const DevPolicy* __restrict__ pol, const int32_t* __restrict__ bundles, DevPlatform plat,
               int64_t nseg, int64_t seg_len, int32_t ngroups, int32_t nbund, StreamWork wk) {
-  constexpr int kStages = Stages<W_T>::n;
+  constexpr int kStages = Stages<W_T, TR>::n;
   constexpr bool kPack = NB > 1;
+  constexpr int kTraces = TR;
+  constexpr int kStageFloats = Cta<TR>::stage_floats;
+  constexpr uint32_t kStageBytes = Cta<TR>::stage_bytes;
+  constexpr int kConsumerWarps = Cta<TR>::consumer_warps;
+  constexpr int kThreads = Cta<TR>::threads;
   extern __shared__ __align__(1024) float sm[];
   __shared__ __align__(8) uint64_t full_bar[kStages];
   __shared__ __align__(8) uint64_t empty_bar[kStages];
@@ -319,6 +349,16 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   const int32_t s = sh_work[0];
   const int32_t bidx = sh_work[1];
   const int32_t g = sh_work[2];
+  if (threadIdx.x == 0) {  // MAGUS_OPT_TRACE: per-CTA timeline
+    if (unsigned long long* tr = trace_buf(wk)) {
+      uint32_t smid;
+      asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+      trace_put(tr, 0, gtimer());
+      trace_put(tr, 4, smid);
+      trace_put(tr, 5, (unsigned long long)s);
+      trace_put(tr, 6, (unsigned long long)g);
+    }
+  }
   int32_t cfg[NB];
 #pragma unroll
   for (int k = 0; k < NB; ++k) cfg[k] = bundles[bidx * NB + k];  // global config, -1 = pad
@@ -347,8 +387,10 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
         if (j >= kStages) mbar_wait(&empty_bar[st], ph ^ 1u);
         mbar_expect_tx(&full_bar[st], kStageBytes + 16u);
         tma_load_1d(st_mul[st], &tmul, &full_bar[st], 2 * (w_first + j));
-        tma_load_2d(sm + st * kStageFloats, &tmap, &full_bar[st], g * kTraces,
-                    (int32_t)((w_first + j) * kRows - wk.tb));
+#pragma unroll
+        for (int b = 0; b < Cta<TR>::boxes; ++b)
+          tma_load_2d(sm + st * kStageFloats + b * (kBox * kRows), &tmap, &full_bar[st], g * kTraces + b * kBox,
+                      (int32_t)((w_first + j) * kRows - wk.tb));
         if (++st == kStages) { st = 0; ph ^= 1u; }
       }
     }
@@ -413,10 +455,12 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
       if (k == kslot) kv = kk[k];
     s_km[kslot][j] = ((kv >> j) & 1) ? ~0u : 0u;
   }
-  consumer_sync();
+  consumer_sync<TR>();
   const uint32_t km_s = smem_u32(&s_km[0][0]);
   const uint32_t full_s = smem_u32(&full_bar[0]), empty_s = smem_u32(&empty_bar[0]);
-  const uint32_t sm_s = smem_u32(sm) + 4u * (uint32_t)tid;  // this thread's column
+  // this thread's column: box tid / 128, lane-in-box tid % 128, row stride 128
+  const int col = TR == kBox ? tid : (tid / kBox) * (kBox * kRows) + (tid % kBox);
+  const uint32_t sm_s = smem_u32(sm) + 4u * (uint32_t)col;
   const uint32_t mul_s = smem_u32(&st_mul[0][0]);
   // words of the trace's last (partial) word and of the warm-up
   const int32_t Ti = (int32_t)T;
@@ -427,7 +471,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   auto word = [&](const int st, const int pst, const uint32_t ph, const int32_t j)
                   __attribute__((always_inline)) {
     mbar_wait_s(full_s + 8u * (uint32_t)st, ph);
-    const float* cur = sm + st * kStageFloats + tid;
+    const float* cur = sm + st * kStageFloats + col;
     const uint32_t cur_s = sm_s + (uint32_t)(st * kStageFloats * 4);
     const int32_t w = w_first + j;
     const int32_t p0 = w * 32;
@@ -439,7 +483,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
       double xd[32];
 #pragma unroll
       for (int i = 0; i < 32; ++i) {
-        const float xi = cur[i * kTraces];
+        const float xi = cur[i * kBox];
         xd[i] = (double)xi;                                    // exact widening, once
         const double xl = (i >= W_T - 1) ? xd[i - (W_T - 1)] : pd[i];
         const double D = xd[i] - xl;                           // Alg. 1 l.3 numerator (RN)
@@ -451,12 +495,12 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
 #pragma unroll
       for (int k = 0; k < W_T - 1; ++k) pd[k] = xd[32 - (W_T - 1) + k];
     } else {
-      const float* prv = sm + pst * kStageFloats + tid;
+      const float* prv = sm + pst * kStageFloats + col;
 #pragma unroll
       for (int i = 0; i < 32; ++i) {
-        const float xi = cur[i * kTraces];
-        const float* b = (i >= W - 1) ? cur : prv + 32 * kTraces;
-        const float xl = b[(i - (W - 1)) * kTraces];
+        const float xi = cur[i * kBox];
+        const float* b = (i >= W - 1) ? cur : prv + 32 * kBox;
+        const float xl = b[(i - (W - 1)) * kBox];
         const double D = (double)xi - (double)xl;
         if (D > d_inc) incw |= 1u << i;
         if (D < d_dec) decw |= 1u << i;
@@ -484,7 +528,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
       uint32_t bb = 0;  // bursts at max uncore: delivered x > theta
       if constexpr (bursts) {
 #pragma unroll
-        for (int i = 0; i < 32; ++i) or_if_gt(bb, cur[i * kTraces], xburst, 1u << i);
+        for (int i = 0; i < 32; ++i) or_if_gt(bb, cur[i * kBox], xburst, 1u << i);
         bb &= outm;
         bbase += __popc(bb);
       }
@@ -646,6 +690,8 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   }
 
   // ---------------- epilogue: publish, look back, correct ----------------
+  if (tid == 0)
+    if (unsigned long long* tr = trace_buf(wk)) trace_put(tr, 1, gtimer());
   {
   // the work coordinates, re-derived from the ticket rather than kept live
   // across the scan (shadowing the names above)
@@ -694,6 +740,8 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
         if (v & 2u) { cin = (v >> 2) & 1u; break; }
       }
     }
+    if (tid == 0 && k == 0)
+      if (unsigned long long* tr = trace_buf(wk)) trace_put(tr, 2, gtimer());
     if (wk.carry && s == nseg - 1)  // no successor reads it: republish as the chunk's final dec
       st_release(status + s * N, (wk.epoch << 3) | 3u | ((seen ? (B.carry >> k) & 1u : cin) << 2));
     uint32_t hi, msr, mdec, mint, ch, bm, pb;
@@ -747,9 +795,9 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
     }
   }
   __threadfence();
-  consumer_sync();
+  consumer_sync<TR>();
   if (tid == 0) sh_last = (atomicAdd(wk.arrive + (int64_t)c0 * ngroups + g, 1u) == (uint32_t)(nseg - 1));
-  consumer_sync();
+  consumer_sync<TR>();
   if (sh_last) {  // all segments of (bundle, group g) are in: finalise the 128 traces
     __threadfence();
 #pragma unroll 1
@@ -791,16 +839,16 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
           for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xFFFFFFFFu, v, o);
           if (lane == 0) sh_red[warp][q] = v;
         }
-        consumer_sync();
+        consumer_sync<TR>();
         if (tid < kTotAcc) {
           unsigned long long v = 0;
           for (int q = 0; q < kConsumerWarps; ++q) v += sh_red[q][tid];
           atomicAdd(wk.tacc + (int64_t)c * kTotAcc + tid, v);
         }
         __threadfence();
-        consumer_sync();
+        consumer_sync<TR>();
         if (tid == 0) sh_last2 = (atomicAdd(wk.tarrive + c, 1u) == (uint32_t)(ngroups - 1));
-        consumer_sync();
+        consumer_sync<TR>();
         if (sh_last2) {
           __threadfence();
           uint64_t* out = wk.totals + (int64_t)c * MAGUS_TOT_WORDS;
@@ -816,11 +864,17 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
             wk.tarrive[c] = 0;
           }
         }
-        consumer_sync();  // sh_red / sh_last2 are reused by the next config
+        consumer_sync<TR>();  // sh_red / sh_last2 are reused by the next config
       }
     }
     if (tid == 0) wk.arrive[(int64_t)c0 * ngroups + g] = 0;
   }
+  }
+  if (tid == 0) {
+    if (unsigned long long* tr = trace_buf(wk)) {
+      trace_put(tr, 3, gtimer());
+      trace_put(tr, 7, sh_last);
+    }
   }
   if (tid == 0) {  // the last CTA of the launch re-arms the ticket counter
     __threadfence();
@@ -837,49 +891,72 @@ typedef void (*stream_fn)(CUtensorMap, CUtensorMap, int64_t, int64_t, const DevP
 struct Pick {
   stream_fn f;
   int smem;
+  int threads;
+  int traces;  // per CTA
 };
 
+template <int W_T, int H_T, int NB, bool BURST, int TR>
+Pick mk() {
+  return {stream_kernel<W_T, H_T, NB, BURST, TR>, Stages<W_T, TR>::smem, Cta<TR>::threads, TR};
+}
+
+// one config per thread with a compile-time W (the paper's H = 10): 512
+// traces per CTA unless `narrow`; everything else 128
 template <int NB, bool BURST>
-Pick pick_nb(int32_t W, int32_t H) {
+Pick pick_nb(int32_t W, int32_t H, bool narrow) {
   if (H == 10) {
+    if constexpr (NB == 1) {
+      if (!narrow) {
+        switch (W) {
+          case 4: return mk<4, 10, NB, BURST, 512>();
+          case 6: return mk<6, 10, NB, BURST, 512>();
+          case 10: return mk<10, 10, NB, BURST, 512>();
+          case 16: return mk<16, 10, NB, BURST, 512>();
+          default: break;
+        }
+      }
+    }
     switch (W) {
-      case 4: return {stream_kernel<4, 10, NB, BURST>, Stages<4>::smem};
-      case 6: return {stream_kernel<6, 10, NB, BURST>, Stages<6>::smem};
-      case 10: return {stream_kernel<10, 10, NB, BURST>, Stages<10>::smem};
-      case 16: return {stream_kernel<16, 10, NB, BURST>, Stages<16>::smem};
+      case 4: return mk<4, 10, NB, BURST, 128>();
+      case 6: return mk<6, 10, NB, BURST, 128>();
+      case 10: return mk<10, 10, NB, BURST, 128>();
+      case 16: return mk<16, 10, NB, BURST, 128>();
       default: break;
     }
-    if (W >= 2 && W <= 33) return {stream_kernel<0, 10, NB, BURST>, Stages<0>::smem};
+    if (W >= 2 && W <= 33) return mk<0, 10, NB, BURST, 128>();
   }
-  if (W >= 2 && W <= 33 && H >= 1 && H <= 32) return {stream_kernel<0, 0, NB, BURST>, Stages<0>::smem};
-  return {nullptr, 0};
+  if (W >= 2 && W <= 33 && H >= 1 && H <= 32) return mk<0, 0, NB, BURST, 128>();
+  return {nullptr, 0, 0, 0};
 }
 
 // The Sec. 6.3 burst counters are a compile-time flag so that the default
 // path carries none of their registers.
-Pick pick(int32_t W, int32_t H, int32_t NB, bool burst = false) {
+Pick pick(int32_t W, int32_t H, int32_t NB, bool burst, bool narrow) {
   switch (NB * 2 + (burst ? 1 : 0)) {
-    case 2: return pick_nb<1, false>(W, H);
-    case 3: return pick_nb<1, true>(W, H);
-    case 4: return pick_nb<2, false>(W, H);
-    case 5: return pick_nb<2, true>(W, H);
-    case 8: return pick_nb<4, false>(W, H);
-    case 9: return pick_nb<4, true>(W, H);
-    default: return {nullptr, 0};
+    case 2: return pick_nb<1, false>(W, H, narrow);
+    case 3: return pick_nb<1, true>(W, H, narrow);
+    case 4: return pick_nb<2, false>(W, H, narrow);
+    case 5: return pick_nb<2, true>(W, H, narrow);
+    case 8: return pick_nb<4, false>(W, H, narrow);
+    case 9: return pick_nb<4, true>(W, H, narrow);
+    default: return {nullptr, 0, 0, 0};
   }
 }
 
 }  // namespace
 
-bool stream_supported(int32_t W, int32_t H) { return pick(W, H, 1).f != nullptr; }
+bool stream_supported(int32_t W, int32_t H) { return pick(W, H, 1, false, false).f != nullptr; }
 
-int stream_ctas_per_sm(int32_t W, int32_t H, int32_t NB) {
-  Pick p = pick(W, H, NB);
+int stream_cta_traces(int32_t W, int32_t H, int32_t NB, bool burst, bool narrow) {
+  return pick(W, H, NB, burst, narrow).traces;
+}
+
+int stream_ctas_per_sm(int32_t W, int32_t H, int32_t NB, bool burst, bool narrow) {
+  Pick p = pick(W, H, NB, burst, narrow);
   if (!p.f) return 0;
   cudaFuncSetAttribute((const void*)p.f, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem);
   int nb = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, (const void*)p.f, kThreads, p.smem) !=
-      cudaSuccess)
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, (const void*)p.f, p.threads, p.smem) != cudaSuccess)
     return 0;
   return nb;
 }
@@ -887,17 +964,17 @@ int stream_ctas_per_sm(int32_t W, int32_t H, int32_t NB) {
 int launch_stream(cudaStream_t st, const void* tmap, const void* tmap_mul, int64_t N, int64_t T,
                   const DevPolicy* pol_dev, const int32_t* bundles_dev, int32_t nbund, int32_t NB,
                   int32_t W, int32_t H, const DevPlatform& plat, int64_t nseg, int64_t seg_len,
-                  const StreamWork& wk, int* grid_out) {
-  Pick p = pick(W, H, NB, plat.burst_on != 0);
+                  const StreamWork& wk, bool narrow, int* grid_out) {
+  Pick p = pick(W, H, NB, plat.burst_on != 0, narrow);
   if (!p.f) return -1;
   cudaFuncSetAttribute((const void*)p.f, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem);
-  const int32_t ngroups = (int32_t)((N + kTraces - 1) / kTraces);
+  const int32_t ngroups = (int32_t)((N + p.traces - 1) / p.traces);
   const int64_t grid = (int64_t)ngroups * nseg * nbund;
   if (grid_out) *grid_out = (int)grid;
   const CUtensorMap* m = reinterpret_cast<const CUtensorMap*>(tmap);
   const CUtensorMap* mm = reinterpret_cast<const CUtensorMap*>(tmap_mul);
-  p.f<<<(unsigned)grid, kThreads, p.smem, st>>>(*m, *mm, N, T, pol_dev, bundles_dev, plat, nseg, seg_len,
-                                                ngroups, nbund, wk);
+  p.f<<<(unsigned)grid, p.threads, p.smem, st>>>(*m, *mm, N, T, pol_dev, bundles_dev, plat, nseg, seg_len,
+                                                 ngroups, nbund, wk);
   return cudaGetLastError() == cudaSuccess ? 1 : -1;
 }
 

@@ -78,6 +78,10 @@ struct StreamWork {
   // is kept (not self-cleaned).
   uint32_t* carry;
 };
+// MAGUS_OPT_TRACE: the per-CTA timeline buffer's address lives in scratch
+// right after the ticket words (ticket[2..3] as a u64, NULL = off), so the
+// kernel's parameter block -- and its register allocation -- is unchanged.
+constexpr int kTraceSlotWords = 2;
 // resume state layout: acc [C][kAccFields][N] u64, then carry [C][N] u32
 inline size_t resume_state_bytes(int64_t N, int32_t C) {
   return 8 * (size_t)kAccFields * (size_t)C * (size_t)N + 4 * (size_t)C * (size_t)N;
@@ -147,8 +151,9 @@ int launch_stream(cudaStream_t s, const void* tmap /* CUtensorMap, host copy */,
                   const void* tmap_mul /* CUtensorMap over StreamWork::mul */, int64_t N,
                   int64_t T, const DevPolicy* pol_dev, const int32_t* bundles_dev, int32_t nbund,
                   int32_t NB, int32_t W, int32_t H, const DevPlatform& plat, int64_t nseg,
-                  int64_t seg_len, const StreamWork& wk, int* grid_out);
-int stream_ctas_per_sm(int32_t W, int32_t H, int32_t NB);
+                  int64_t seg_len, const StreamWork& wk, bool narrow, int* grid_out);
+int stream_ctas_per_sm(int32_t W, int32_t H, int32_t NB, bool burst, bool narrow);
+int stream_cta_traces(int32_t W, int32_t H, int32_t NB, bool burst, bool narrow);  // traces per CTA
 
 // NEXT f2 DP (kernels_bound.cu): out [N][nl][3] = {cost, energy, time}.
 int launch_bound(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,

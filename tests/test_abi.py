@@ -100,10 +100,11 @@ def _consumer_loop_local_ops(sass: str):
     return hi - lo, [hex(a) for a, t in ins if lo <= a <= hi and ("STL" in t or "LDL" in t)]
 
 
-@pytest.mark.parametrize("inst,budget", [("ILi10ELi10ELi1ELb0E", 0), ("ILi10ELi10ELi4ELb0E", 2),
-                                         ("ILi4ELi10ELi4ELb0E", 2)])
+@pytest.mark.parametrize("inst,budget", [("ILi10ELi10ELi1ELb0ELi512E", 0), ("ILi10ELi10ELi4ELb0ELi128E", 2),
+                                         ("ILi4ELi10ELi4ELb0ELi128E", 2)])
 def test_hot_kernels_do_not_spill_in_the_word_loop(inst, budget):
-    """The paper-default kernel (W = H = 10, one config per thread) keeps its
+    """The paper-default kernel (W = H = 10, one config per thread, 512-trace
+    CTAs) keeps its
     whole word loop in registers; the 4-config bundle kernels of SWEEP256 may
     reload at most two loop-invariant words per 32-step word (~1000
     instructions).  A few bytes spilled around the loop are harmless."""

@@ -68,12 +68,13 @@ def test_bench_steps_in_flight_agree(config):
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     lines = []
     for inflight in (1, 2):
-        r = subprocess.run([sys.executable, "bench.py", "--config", str(config), "--n-traces", "256", "--n-steps",
-                            "4000", "--steps", "6", "--warmup", "3", "--no-cpu-baseline", "--no-e2e",
+        r = subprocess.run([sys.executable, "bench.py", "--config", str(config), "--n-traces", "1024", "--n-steps",
+                            "131072", "--steps", "6", "--warmup", "3", "--no-cpu-baseline", "--no-e2e",
                             "--inflight", str(inflight)], cwd=root, capture_output=True, text=True, timeout=600)
         assert r.returncode == 0, r.stderr[-2000:]
         lines.append(json.loads(r.stdout.strip().splitlines()[-1]))
     a, b = lines
-    assert a["config"]["steps_in_flight"] == 1 and b["config"]["steps_in_flight"] == 2
+    # (inputs above 4 x L2: no flush between steps, so steps may overlap)
+    assert a["run"]["steps_in_flight"] == 1 and b["run"]["steps_in_flight"] == 2
     assert a["best_config"] == b["best_config"] and a["feasible"] == b["feasible"]
     assert a["gpu_launches"] == b["gpu_launches"]
