@@ -111,107 +111,6 @@ __device__ __forceinline__ double q_as_double(double xd, double invB) {
   return r > 1.0 ? s24 : 0.0;
 }
 
-// The full ratio grid with a compile-time level count L (the platforms'
-// 15 and 18 ratios): every per-level array is register-resident (fully
-// unrolled loops; the chosen predecessor's energy / time are picked by
-// selects, not by a dynamic index), in-place update.  Same fp64 operations
-// in the same order as bound_kernel.
-template <int L>
-__global__ void __launch_bounds__(kBoundThreads)
-bound_grid_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
-                  const double* __restrict__ lambdas, int32_t nl, DevPlatform plat, double bw_max,
-                  double p_lo, double p_span, double* __restrict__ out) {
-  __shared__ double s_invB[L], s_P[L];
-  __shared__ float s_x[32][kBoundThreads];
-  for (int i = threadIdx.x; i < L; i += blockDim.x) {
-    const int l = plat.r_min + i;
-    const double B = (bw_max * (double)l) / (double)plat.r_max;
-    s_invB[i] = 1.0 / B;
-    s_P[i] = p_lo + (p_span * (double)(l - plat.r_min)) / (double)(plat.r_max - plat.r_min);
-  }
-  __syncthreads();
-  const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const bool active = gid < N * nl;
-  const int32_t j = active ? (int32_t)(gid / N) : 0;
-  const int64_t n = active ? gid - (int64_t)j * N : 0;
-  const double lam = lambdas[j];
-  const double sw_c = plat.e_sw + lam * plat.t_sw;
-  constexpr int imax = L - 1;  // ascending level set ending at r_max
-
-  double V[L], E[L], Tm[L];
-#pragma unroll
-  for (int i = 0; i < L; ++i) { V[i] = INFINITY; E[i] = 0.0; Tm[i] = 0.0; }
-
-  for (int64_t t = 0; t < T; ++t) {
-    const int jj = (int)(t & 31);
-    if (jj == 0) {  // stage the next 32 samples of this trace (independent loads)
-      __syncwarp();
-#pragma unroll 8
-      for (int i = 0; i < 32; ++i)
-        s_x[i][threadIdx.x] = (active && t + i < T) ? x[(t + i) * ld + n] : 0.0f;
-      __syncwarp();
-    }
-    const float xt = s_x[jj][threadIdx.x];
-    const double xd = (double)xt;
-    if (t == 0) {
-      const double tau = plat.dt + plat.cQ * q_as_double(xd, s_invB[imax]);
-      const double e = s_P[imax] * tau;
-      V[imax] = e + lam * tau;
-      E[imax] = e;
-      Tm[imax] = tau;
-      continue;
-    }
-    // best and second best previous state (lowest index on ties)
-    int a1 = 0;
-    double m1 = V[0];
-#pragma unroll
-    for (int i = 1; i < L; ++i)
-      if (V[i] < m1) { m1 = V[i]; a1 = i; }
-    int a2 = -1;
-    double m2 = INFINITY;
-#pragma unroll
-    for (int i = 0; i < L; ++i)
-      if (i != a1 && (a2 < 0 || V[i] < m2)) { m2 = V[i]; a2 = i; }
-    double E1 = 0.0, T1 = 0.0, E2 = 0.0, T2 = 0.0;
-#pragma unroll
-    for (int i = 0; i < L; ++i) {
-      if (i == a1) { E1 = E[i]; T1 = Tm[i]; }
-      if (i == a2) { E2 = E[i]; T2 = Tm[i]; }
-    }
-    const bool sw = t >= 2;
-#pragma unroll
-    for (int i = 0; i < L; ++i) {
-      const bool isa1 = i == a1;
-      const double other = isa1 ? m2 : m1;
-      const double move = sw ? other + sw_c : other;
-      double v, e0, t0;
-      if (V[i] <= move) {
-        v = V[i]; e0 = E[i]; t0 = Tm[i];
-      } else {
-        const double Eo = isa1 ? E2 : E1, To = isa1 ? T2 : T1;
-        v = move;
-        e0 = sw ? Eo + plat.e_sw : Eo;
-        t0 = sw ? To + plat.t_sw : To;
-      }
-      const double tau = plat.dt + plat.cQ * q_as_double(xd, s_invB[i]);
-      const double e = s_P[i] * tau;
-      V[i] = v + (e + lam * tau);
-      E[i] = e0 + e;
-      Tm[i] = t0 + tau;
-    }
-  }
-  if (!active) return;
-  int b = 0;
-  double vb = V[0], eb = E[0], tb = Tm[0];
-#pragma unroll
-  for (int i = 1; i < L; ++i)
-    if (V[i] < vb) { b = i; vb = V[i]; eb = E[i]; tb = Tm[i]; }
-  double* o = out + ((int64_t)n * nl + j) * 3;
-  o[0] = vb;
-  o[1] = eb;
-  o[2] = tb;
-}
-
 // The binary level set {r_min, r_max}: the same recurrence with the two
 // states in scalar registers (the generic kernel's arrays live in local
 // memory) and the samples of 32 intervals loaded ahead.  For L = 2 the
@@ -282,22 +181,498 @@ bound_binary_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t l
   o[2] = b1 ? T1 : T0;
 }
 
+
+// ---------------------------------------------------------------------------
+// bound_dp_kernel<L>: the same DP, restructured for throughput.
+// Every result is bit-identical to bound_kernel / the oracle DP: the same fp64
+// operations on the same operands in the same order; only which of them are
+// evaluated, and where the operands are kept, changes.
+//
+// * No second minimum.  The move candidate of level i is the lowest-index
+//   minimum a1 of the previous values for every i != a1, and a1 itself always
+//   stays: V[a1] = m1 <= V[o] <= RN(V[o] + sw_c) for any other o, because
+//   sw_c = e_sw + lambda * t_sw >= 0 (validated finite and >= 0, so no NaN)
+//   and RN is monotone.  So every level compares against ONE move value
+//   mv = m1 (+ sw_c) and inherits (E1, T1) = (E, T)[a1] when it moves.
+// * Two passes per 32-step chunk.  Pass 1 runs the value chain only (V per
+//   level, the lowest-index minimum, which levels stayed); pass 2 the path
+//   sums.  When no level other than a1 stays in a step (always, up to exact
+//   ties, when switches are free: e_sw = t_sw = 0, the paper's "negligible"
+//   MSR writes), every level's new (E, T) is (E1, T1) or (Eb, Tb) plus its
+//   own (e, tau), so only (E1, T1) are followed: E1' = (a1' == a1 ? E1 : Eb)
+//   + e[a1'] (mode A).  A step where another level stays (a tie, or
+//   sw_c > 0) keeps per-level (E, T) (mode B), rebuilt first from the last
+//   mode-A step's record (its sample, the level that stayed, the two bases)
+//   -- again the operations the oracle did.  Modes are warp-uniform.
+// * Two lanes per (trace, lambda) chain, each owning half of the levels
+//   (16 chains per warp), so a sub-partition holds ~2 warps of independent
+//   work; a chain's minimum is its lanes' local trees merged by one shuffle
+//   (the lower half wins ties: the lowest-index rule).
+// * Stretch work only where it exists: the thresholds x*_l (x > x*_l <=>
+//   RN(x * invB_l) > 1, host-inverted) rise with the level, so the levels with
+//   a stretch at step t are a prefix [0, s) (warp max).  Their costs are
+//   written to a per-lane row in shared memory; otherwise the q = 0 costs
+//   (tau = dt, e = P_l * dt, e + lambda * dt: the same operations with q = 0)
+//   are register constants.
+// * Lanes are (trace, lambda) with lambda fastest; one warp per CTA; a rolled
+//   step loop; samples staged per warp by cp.async, double-buffered.
+// ---------------------------------------------------------------------------
+struct BoundThr {
+  float x[32];  // x*_l per level of the DP's level set (stretch_threshold)
+};
+
+constexpr int kDpChunk = 32;
+
+__device__ __forceinline__ void cp_async4(float* dst, const float* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(dst)),
+               "l"(src)
+               : "memory");
+}
+
+// V' = (V <= mv ? V : mv) + c, stay bit `bit` set when V <= mv
+__device__ __forceinline__ void v_update(double& v, uint32_t& stay, double mv, uint32_t bit, double c) {
+  asm("{\n.reg .pred p;\n"
+      "setp.le.f64 p, %0, %2;\n"
+      "@p or.b32 %1, %1, %3;\n"
+      "selp.f64 %0, %0, %2, p;\n"
+      "add.rn.f64 %0, %0, %4;\n}"
+      : "+d"(v), "+r"(stay)
+      : "d"(mv), "r"(bit), "d"(c));
+}
+
+template <int L>
+__global__ void __launch_bounds__(32)
+bound_dp_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
+                const double* __restrict__ lambdas, int32_t nl, int32_t lstep, DevPlatform plat,
+                double bw_max, double p_lo, double p_span, const __grid_constant__ BoundThr thr,
+                double* __restrict__ out) {
+  static_assert(L >= 4 && L <= 18, "level set");
+  constexpr int H = (L + 1) / 2;  // levels per lane: [0, H) and [H, L)
+  __shared__ double s_invB[2 * H], s_P[2 * H], s_Pdt[2 * H];
+  __shared__ double s_c[H * 32];  // [local level][lane]: this step's stretched costs
+  __shared__ float s_thr[32];
+  __shared__ float s_x[2][kDpChunk][32];
+  __shared__ uint8_t s_a1[kDpChunk][32];    // pass 1 -> 2: argmin of each step
+  __shared__ uint32_t s_stay[kDpChunk][32];  // pass 1 -> 2: this lane's levels that stayed
+  const int lane = threadIdx.x;
+  const int h = lane & 1;          // which half of the levels
+  const int base = h * H;          // first level of this lane
+  for (int i = lane; i < 2 * H; i += 32) {
+    if (i < L) {
+      const int l = plat.r_min + i * lstep;
+      const double B = (bw_max * (double)l) / (double)plat.r_max;
+      s_invB[i] = 1.0 / B;
+      s_P[i] = p_lo + (p_span * (double)(l - plat.r_min)) / (double)(plat.r_max - plat.r_min);
+      s_Pdt[i] = s_P[i] * plat.dt;  // e at q = 0: P_l * (dt + cQ * 0) = P_l * dt
+    } else {  // the padding level of an odd L: never reachable
+      s_invB[i] = 0.0;
+      s_P[i] = 0.0;
+      s_Pdt[i] = 0.0;
+    }
+  }
+  s_thr[lane] = lane < L ? thr.x[lane] : INFINITY;
+  __syncwarp();
+  const int64_t chain = (int64_t)blockIdx.x * 16 + (lane >> 1);
+  const bool active = chain < N * nl;
+  const int64_t n = active ? chain / nl : 0;
+  const int32_t j = active ? (int32_t)(chain - n * nl) : 0;
+  const double lam = lambdas[j];
+  const double dt = plat.dt, cQ = plat.cQ, e_sw = plat.e_sw, t_sw = plat.t_sw;
+  const double sw_c = e_sw + lam * t_sw;
+  const double lt0 = lam * dt;  // lambda * tau at q = 0
+  double cf[H];                 // this lane's costs at q = 0 (+inf: the padding level)
+#pragma unroll
+  for (int i = 0; i < H; ++i) cf[i] = (base + i < L) ? s_Pdt[base + i] + lt0 : INFINITY;
+
+  double V[H], E[H], Tm[H];
+  const float* px = x + n;
+  // t = 0: every level's (e, tau); only r_max (the last level) is reachable
+  {
+    const double xd = (double)(active ? __ldg(px) : 0.0f);
+#pragma unroll
+    for (int i = 0; i < H; ++i) {
+      const int g = base + i;
+      const double tau = dt + cQ * q_as_double(xd, s_invB[g]);
+      const double e = s_P[g] * tau;
+      V[i] = (g == L - 1) ? e + lam * tau : INFINITY;
+      E[i] = e;
+      Tm[i] = tau;
+    }
+  }
+  // the chain's scalars (identical in both lanes)
+  double m1, E1, T1;
+  {
+    const int o = (L - 1) - H;  // r_max is local level L-1-H of the upper lane
+    const double v = h ? V[o] : 0.0, e = h ? E[o] : 0.0, t = h ? Tm[o] : 0.0;
+    m1 = __shfl_sync(0xFFFFFFFFu, v, lane | 1);
+    E1 = __shfl_sync(0xFFFFFFFFu, e, lane | 1);
+    T1 = __shfl_sync(0xFFFFFFFFu, t, lane | 1);
+  }
+  int a1 = L - 1;
+  bool inB = true;  // the per-level (E, T) arrays are current
+  // mode-A record of the last step: its sample, the level that stayed, the bases
+  double r_x = 0.0, r_E1 = 0.0, r_Eb = 0.0, r_T1 = 0.0, r_Tb = 0.0;
+  int r_a1 = L - 1;
+  int prev_ns = 0;  // the last step stretched levels [0, prev_ns)
+  // samples t = 1 + c * 32 + k in chunk c, staged into s_x[c & 1][k][lane]
+  const int64_t nch = (T - 1 + kDpChunk - 1) / kDpChunk;
+  auto stage = [&](int64_t c) {
+    const int64_t t0 = 1 + c * kDpChunk;
+    const int kmax = (int)(T - t0 < kDpChunk ? T - t0 : kDpChunk);
+    const float* src = px + (active ? t0 * ld : 0);
+    const int64_t step = active ? ld : 0;
+    float* dst = &s_x[c & 1][0][lane];
+#pragma unroll 8
+    for (int k = 0; k < kmax; ++k) {
+      cp_async4(dst + k * 32, src);
+      src += step;
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  if (nch > 0) stage(0);
+  for (int64_t c = 0; c < nch; ++c) {
+    if (c + 1 < nch) {
+      stage(c + 1);
+      asm volatile("cp.async.wait_group 1;" ::: "memory");
+    } else {
+      asm volatile("cp.async.wait_group 0;" ::: "memory");
+    }
+    __syncwarp();
+    const int64_t t0 = 1 + c * kDpChunk;
+    const int kn = (int)(T - t0 < kDpChunk ? T - t0 : kDpChunk);
+    const float* xs = &s_x[c & 1][0][lane];
+    // ---- pass 1: the value chain (V per level, m1, argmin, stay bits) ----
+#pragma unroll 1
+    for (int k = 0; k < kn; ++k) {
+      const bool sw = t0 + k >= 2;
+      const double mv = sw ? m1 + sw_c : m1;
+      const float xf = xs[k * 32];
+      // levels with a stretch at this step: a prefix [0, ns) (NaN: none)
+      int ns = 0;
+      if (__any_sync(0xFFFFFFFFu, xf > s_thr[0])) {
+#pragma unroll
+        for (int w = 16; w > 0; w >>= 1)
+          if (ns + w <= L && xf > s_thr[ns + w - 1]) ns += w;
+        ns = __reduce_max_sync(0xFFFFFFFFu, ns);
+      }
+      uint32_t stay = 0;
+      if (ns == 0) {  // every cost is its q = 0 constant
+#pragma unroll
+        for (int i = 0; i < H; ++i) v_update(V[i], stay, mv, 1u << i, cf[i]);
+      } else {
+        // this lane's stretched levels [base, ns) get the full model-M cost
+        const double xd = (double)xf;
+        const int nloc = ns - base;
+#pragma unroll 1
+        for (int i = 0; i < nloc && i < H; ++i) {
+          const double tau = dt + cQ * q_as_double(xd, s_invB[base + i]);
+          const double e = s_P[base + i] * tau;
+          s_c[i * 32 + lane] = e + lam * tau;
+        }
+#pragma unroll
+        for (int i = 0; i < H; ++i) v_update(V[i], stay, mv, 1u << i, i < nloc ? s_c[i * 32 + lane] : cf[i]);
+      }
+      (void)prev_ns;
+      // lowest-index minimum: local pairwise tree, then the two halves
+      double tv[H];
+      int ti[H];
+#pragma unroll
+      for (int i = 0; i < H; ++i) { tv[i] = V[i]; ti[i] = base + i; }
+#pragma unroll
+      for (int w = 1; w < H; w *= 2) {
+#pragma unroll
+        for (int i = 0; i + w < H; i += 2 * w) {
+          const bool r = tv[i + w] < tv[i];
+          tv[i] = r ? tv[i + w] : tv[i];
+          ti[i] = r ? ti[i + w] : ti[i];
+        }
+      }
+      const double vo = __shfl_xor_sync(0xFFFFFFFFu, tv[0], 1);
+      const int io = __shfl_xor_sync(0xFFFFFFFFu, ti[0], 1);
+      // the partner wins if strictly smaller, or equal and lower (h = 1 takes an equal lower half)
+      const bool take = h ? (vo <= tv[0]) : (vo < tv[0]);
+      m1 = take ? vo : tv[0];
+      s_a1[k][lane] = (uint8_t)(take ? io : ti[0]);
+      s_stay[k][lane] = stay;
+    }
+    // ---- pass 2: the path sums (E, T) along the chosen predecessors ----
+    // A step where a level other than the previous argmin stayed needs the
+    // per-level histories (mode B); find out for the whole chunk first
+    uint32_t other = 0;
+    {
+      int pa = a1;
+#pragma unroll 1
+      for (int k = 0; k < kn; ++k) {
+        const int lb = pa - base;  // the argmin's bit in this lane's mask, if it is here
+        other |= s_stay[k][lane] & ~((lb >= 0 && lb < H) ? (1u << lb) : 0u);
+        pa = s_a1[k][lane];
+      }
+    }
+    if (!__any_sync(0xFFFFFFFFu, other != 0u)) {
+      // mode A throughout: every level but the argmin moved, so (E1, T1)
+      // follow the argmin: E1' = (a1' == a1 ? E1 : Eb) + e[a1']
+      double pE1 = E1, pEb = E1, pT1 = T1, pTb = T1, px_ = r_x;
+      int pa1 = a1;
+#pragma unroll 4
+      for (int k = 0; k < kn; ++k) {
+        const bool sw = t0 + k >= 2;
+        const double Eb = sw ? E1 + e_sw : E1;
+        const double Tb = sw ? T1 + t_sw : T1;
+        const int na = s_a1[k][lane];
+        const double xd = (double)xs[k * 32];
+        const double tau_a = dt + cQ * q_as_double(xd, s_invB[na]);  // q = 0: dt, P * dt
+        const double e_a = s_P[na] * tau_a;
+        pE1 = E1; pEb = Eb; pT1 = T1; pTb = Tb; px_ = xd; pa1 = a1;
+        E1 = (na == a1 ? E1 : Eb) + e_a;
+        T1 = (na == a1 ? T1 : Tb) + tau_a;
+        a1 = na;
+      }
+      if (kn > 0) {
+        r_x = px_; r_a1 = pa1; r_E1 = pE1; r_Eb = pEb; r_T1 = pT1; r_Tb = pTb;
+        inB = false;
+      }
+    } else {
+#pragma unroll 1
+      for (int k = 0; k < kn; ++k) {
+        const bool sw = t0 + k >= 2;
+        const double Eb = sw ? E1 + e_sw : E1;
+        const double Tb = sw ? T1 + t_sw : T1;
+        const int na = s_a1[k][lane];
+        const uint32_t stay = s_stay[k][lane];
+        const double xd = (double)xs[k * 32];
+        const int lb = a1 - base;
+        if (__any_sync(0xFFFFFFFFu, (stay & ~((lb >= 0 && lb < H) ? (1u << lb) : 0u)) != 0u)) {
+          // mode B: per-level (E, T)
+          if (!inB) {  // rebuild (E, T) of the last step from its record
+#pragma unroll
+            for (int i = 0; i < H; ++i) {
+              const double tau = dt + cQ * q_as_double(r_x, s_invB[base + i]);
+              const double e = s_P[base + i] * tau;
+              E[i] = (base + i == r_a1 ? r_E1 : r_Eb) + e;
+              Tm[i] = (base + i == r_a1 ? r_T1 : r_Tb) + tau;
+            }
+            inB = true;
+          }
+          double eo = 0.0, to = 0.0;
+#pragma unroll
+          for (int i = 0; i < H; ++i) {
+            const double tau = dt + cQ * q_as_double(xd, s_invB[base + i]);
+            const double e = s_P[base + i] * tau;
+            const bool st = (stay >> i) & 1u;
+            E[i] = (st ? E[i] : Eb) + e;
+            Tm[i] = (st ? Tm[i] : Tb) + tau;
+            if (base + i == na) { eo = E[i]; to = Tm[i]; }
+          }
+          const int owner = (lane & ~1) | (na >= H ? 1 : 0);
+          E1 = __shfl_sync(0xFFFFFFFFu, eo, owner);
+          T1 = __shfl_sync(0xFFFFFFFFu, to, owner);
+        } else {
+          const double tau_a = dt + cQ * q_as_double(xd, s_invB[na]);
+          const double e_a = s_P[na] * tau_a;
+          r_x = xd; r_a1 = a1; r_E1 = E1; r_Eb = Eb; r_T1 = T1; r_Tb = Tb;
+          E1 = (na == a1 ? E1 : Eb) + e_a;
+          T1 = (na == a1 ? T1 : Tb) + tau_a;
+          inB = false;
+        }
+        a1 = na;
+      }
+    }
+    __syncwarp();  // s_x[c & 1] is restaged by chunk c + 2
+  }
+  if (!active || h) return;
+  double* o = out + chain * 3;  // [n][nl][3]: chain = n * nl + j
+  o[0] = m1;
+  o[1] = E1;
+  o[2] = T1;
+}
+
+// ---------------------------------------------------------------------------
+// bound_binary_free_kernel: the binary DP when switches are free (e_sw =
+// t_sw = 0, the paper's "negligible" MSR writes -- the default platform).
+// Then mv = m1 and a level stays only if V == m1, so without a tie every
+// level's new value is m1 + c (stay or move alike: V = m1 when it stays),
+// the new minimum is the smaller sum (the lower level on equality), and the
+// path sums follow the argmin: E1 += e[a1'], T1 += tau[a1'] (Eb = E1 + 0 =
+// E1).  Per step: two adds, a compare, three selects and two adds.  A tie
+// (s0 == s1: both levels minimal) gives the levels different histories, so
+// the warp rebuilds the per-level state of that step -- V_i = s_i,
+// E_i = E1 + e_i, T_i = T1 + tau_i, the oracle's own sums -- and finishes
+// with the general per-level recurrence (bound_binary_kernel's step).
+// Lanes are (trace, lambda) with lambda fastest, so the stretch branch (a
+// warp-wide vote on x > x*_min, host-inverted) is rarely taken; samples are
+// staged per warp by cp.async, double-buffered; one warp per CTA.
+// ---------------------------------------------------------------------------
+constexpr int kBinChunk = 32;  // steps per staged chunk
+
+__global__ void __launch_bounds__(32)
+bound_binary_free_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
+                         const double* __restrict__ lambdas, int32_t nl, DevPlatform plat, double bw_max,
+                         double p_lo, double p_span, float xthr0, double* __restrict__ out) {
+  __shared__ float s_x[2][kBinChunk][32];
+  const int lane = threadIdx.x;
+  const int64_t gid = (int64_t)blockIdx.x * 32 + lane;
+  const bool active = gid < N * nl;
+  const int64_t n = active ? gid / nl : 0;
+  const int32_t j = active ? (int32_t)(gid - n * nl) : 0;
+  const double lam = lambdas[j];
+  const int lmin = plat.r_min, lmax = plat.r_max;
+  const double invB0 = 1.0 / ((bw_max * (double)lmin) / (double)lmax);
+  const double invB1 = 1.0 / ((bw_max * (double)lmax) / (double)lmax);
+  const double P0 = p_lo + (p_span * (double)(lmin - lmin)) / (double)(lmax - lmin);
+  const double P1 = p_lo + (p_span * (double)(lmax - lmin)) / (double)(lmax - lmin);
+  const double dt = plat.dt, cQ = plat.cQ;
+  const double Pdt0 = P0 * dt, Pdt1 = P1 * dt;         // e at q = 0
+  const double cf0 = Pdt0 + lam * dt, cf1 = Pdt1 + lam * dt;  // e + lambda * tau at q = 0
+  const float* px = x + n;
+  // t = 0 runs at r_max
+  double m1, E1, T1;
+  {
+    const double xd = (double)(active ? __ldg(px) : 0.0f);
+    const double tau1 = dt + cQ * q_as_double(xd, invB1);
+    const double e1 = P1 * tau1;
+    m1 = e1 + lam * tau1;
+    E1 = e1;
+    T1 = tau1;
+  }
+  bool general = false;  // warp-uniform: per-level recurrence after a tie
+  double V0 = 0.0, V1 = 0.0, E0 = 0.0, Ea = 0.0, T0 = 0.0, Ta = 0.0;  // its per-level state
+  const int64_t nch = (T - 1 + kBinChunk - 1) / kBinChunk;
+  auto stage = [&](int64_t c) {
+    const int64_t t0 = 1 + c * kBinChunk;
+    const int kmax = (int)(T - t0 < kBinChunk ? T - t0 : kBinChunk);
+    const float* src = px + (active ? t0 * ld : 0);
+    const int64_t step = active ? ld : 0;
+    float* dst = &s_x[c & 1][0][lane];
+#pragma unroll 8
+    for (int k = 0; k < kmax; ++k) {
+      cp_async4(dst + k * 32, src);
+      src += step;
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  if (nch > 0) stage(0);
+  for (int64_t c = 0; c < nch; ++c) {
+    if (c + 1 < nch) {
+      stage(c + 1);
+      asm volatile("cp.async.wait_group 1;" ::: "memory");
+    } else {
+      asm volatile("cp.async.wait_group 0;" ::: "memory");
+    }
+    __syncwarp();
+    const int64_t t0 = 1 + c * kBinChunk;
+    const int kn = (int)(T - t0 < kBinChunk ? T - t0 : kBinChunk);
+    const float* xs = &s_x[c & 1][0][lane];
+    // (c, e, tau) of both levels at a sample: full model M
+    auto costs = [&](float xf, double& c0, double& c1, double& e0, double& e1, double& tau0, double& tau1) {
+      const double xd = (double)xf;
+      tau0 = dt + cQ * q_as_double(xd, invB0);
+      tau1 = dt + cQ * q_as_double(xd, invB1);
+      e0 = P0 * tau0;
+      e1 = P1 * tau1;
+      c0 = e0 + lam * tau0;
+      c1 = e1 + lam * tau1;
+    };
+    bool redo = false;
+    if (!general) {
+      // fast sweep over the chunk; a tie anywhere sends the warp back to the
+      // chunk's start for the careful sweep below
+      const double m1s = m1, E1s = E1, T1s = T1;
+      bool tie = false;
+#pragma unroll 4
+      for (int k = 0; k < kn; ++k) {
+        const float xf = xs[k * 32];
+        if (__any_sync(0xFFFFFFFFu, xf > xthr0)) {  // some lane has a stretch
+          double c0, c1, e0, e1, tau0, tau1;
+          costs(xf, c0, c1, e0, e1, tau0, tau1);
+          const double s0 = m1 + c0, s1 = m1 + c1;
+          tie |= s0 == s1;
+          const bool up = s1 < s0;
+          m1 = up ? s1 : s0;
+          E1 = E1 + (up ? e1 : e0);
+          T1 = T1 + (up ? tau1 : tau0);
+        } else {
+          const double s0 = m1 + cf0, s1 = m1 + cf1;
+          tie |= s0 == s1;
+          const bool up = s1 < s0;
+          m1 = up ? s1 : s0;
+          E1 = E1 + (up ? Pdt1 : Pdt0);
+          T1 = T1 + dt;
+        }
+      }
+      if (__any_sync(0xFFFFFFFFu, tie)) {
+        m1 = m1s; E1 = E1s; T1 = T1s;
+        redo = true;
+      }
+    }
+    if (general || redo) {
+#pragma unroll 1
+      for (int k = 0; k < kn; ++k) {
+        double c0, c1, e0, e1, tau0, tau1;
+        costs(xs[k * 32], c0, c1, e0, e1, tau0, tau1);
+        if (!general) {
+          const double s0 = m1 + c0, s1 = m1 + c1;
+          if (__any_sync(0xFFFFFFFFu, s0 == s1)) {
+            // a tie: rebuild every lane's per-level state of this step
+            V0 = s0; V1 = s1;
+            E0 = E1 + e0; Ea = E1 + e1;
+            T0 = T1 + tau0; Ta = T1 + tau1;
+            general = true;
+          } else {
+            const bool up = s1 < s0;
+            m1 = up ? s1 : s0;
+            E1 = E1 + (up ? e1 : e0);
+            T1 = T1 + (up ? tau1 : tau0);
+          }
+        } else {  // the general recurrence (free switches: mv = the other level's V)
+          const bool st0 = V0 <= V1, st1 = V1 <= V0;  // stay before move
+          const double nV0 = (st0 ? V0 : V1) + c0, nE0 = (st0 ? E0 : Ea) + e0, nT0 = (st0 ? T0 : Ta) + tau0;
+          const double nV1 = (st1 ? V1 : V0) + c1, nE1 = (st1 ? Ea : E0) + e1, nT1 = (st1 ? Ta : T0) + tau1;
+          V0 = nV0; E0 = nE0; T0 = nT0;
+          V1 = nV1; Ea = nE1; Ta = nT1;
+        }
+      }
+    }
+    __syncwarp();  // s_x[c & 1] is restaged by chunk c + 2
+  }
+  if (general) {
+    const bool b1 = V1 < V0;  // lowest index on ties
+    m1 = b1 ? V1 : V0;
+    E1 = b1 ? Ea : E0;
+    T1 = b1 ? Ta : T0;
+  }
+  if (!active) return;
+  double* o = out + gid * 3;
+  o[0] = m1;
+  o[1] = E1;
+  o[2] = T1;
+}
+
 int launch_bound(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,
                  const double* lambdas_dev, int32_t nl, bool full_grid, const DevPlatform& plat,
                  double bw_max, double p_lo, double p_span, double* out) {
   const int32_t L = full_grid ? plat.r_max - plat.r_min + 1 : 2;
   const int32_t lstep = full_grid ? 1 : plat.r_max - plat.r_min;
   const unsigned blocks = (unsigned)((N * nl + kBoundThreads - 1) / kBoundThreads);
-  if (L == 2)
+  // (every lambda and switch cost is finite and >= 0, validated by the caller)
+  BoundThr thr;
+  for (int i = 0; i < 32; ++i) {
+    const int l = plat.r_min + i * lstep;
+    thr.x[i] = i < L ? stretch_threshold(1.0 / ((bw_max * (double)l) / (double)plat.r_max)) : INFINITY;
+  }
+  const unsigned warps = (unsigned)((N * nl + 15) / 16);  // 16 chains (2 lanes each) per warp
+  if (L == 2 && plat.e_sw == 0.0 && plat.t_sw == 0.0)
+    bound_binary_free_kernel<<<(unsigned)((N * nl + 31) / 32), 32, 0, s>>>(x, N, T, ld, lambdas_dev, nl, plat,
+                                                                         bw_max, p_lo, p_span, thr.x[0], out);
+  else if (L == 2)  // two levels with switch costs: the branch-free per-step kernel
     bound_binary_kernel<<<blocks, kBoundThreads, 0, s>>>(x, N, T, ld, lambdas_dev, nl, plat, bw_max, p_lo,
                                                          p_span, out);
   else if (L == 15)
-    bound_grid_kernel<15><<<blocks, kBoundThreads, 0, s>>>(x, N, T, ld, lambdas_dev, nl, plat, bw_max, p_lo,
-                                                           p_span, out);
+    bound_dp_kernel<15><<<warps, 32, 0, s>>>(x, N, T, ld, lambdas_dev, nl, lstep, plat, bw_max, p_lo, p_span, thr,
+                                             out);
   else if (L == 18)
-    bound_grid_kernel<18><<<blocks, kBoundThreads, 0, s>>>(x, N, T, ld, lambdas_dev, nl, plat, bw_max, p_lo,
-                                                           p_span, out);
-  else
+    bound_dp_kernel<18><<<warps, 32, 0, s>>>(x, N, T, ld, lambdas_dev, nl, lstep, plat, bw_max, p_lo, p_span, thr,
+                                             out);
+  else  // other level counts: the generic kernel
     bound_kernel<32><<<blocks, kBoundThreads, 0, s>>>(x, N, T, ld, lambdas_dev, nl, L, plat.r_min, lstep,
                                                       plat, bw_max, p_lo, p_span, out);
   return cudaGetLastError() == cudaSuccess ? 1 : -1;

@@ -118,3 +118,38 @@ def test_gpu_offline_bound_bit_exact(full_grid, r_max):
         for j, lam in enumerate(lams):
             ref = oracle.offline_bound(x[:, n], lam, plat_o, full_grid=full_grid)
             assert np.array_equal(got[n, j], ref), (n, lam)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("full_grid", [False, True])
+@pytest.mark.parametrize("case", ["free_switch", "flat_power_ties", "tiny_switch", "adversarial", "short"])
+def test_gpu_offline_bound_modes_bit_exact(full_grid, case):
+    """The throughput kernel's two bookkeeping modes: free
+    switches (the paper's default: scalar path sums), equal power at every
+    level (exact ties everywhere: per-level histories and the lowest-index
+    rule), a tiny switch cost (mode changes mid-chunk), adversarial traces,
+    and T = 1, 2, 33, 34 -- all bit for bit against the oracle DP."""
+    torch = pytest.importorskip("torch")
+    magus = pytest.importorskip("paper_conf_sc_zhengspl25_b200")
+    kw = {"free_switch": {}, "flat_power_ties": dict(p_unc_min=41.0, p_unc_max=41.0),
+          "tiny_switch": dict(e_sw=1e-9, p_unc_min=41.0, p_unc_max=41.0000001),
+          "adversarial": dict(e_sw=0.5), "short": {}}[case]
+    plat = magus.platform_preset()
+    plat.e_switch_j = kw.get("e_sw", 0.0)
+    plat.p_unc_min_w = kw.get("p_unc_min", plat.p_unc_min_w)
+    plat.p_unc_max_w = kw.get("p_unc_max", plat.p_unc_max_w)
+    plat_o = oracle.platform(**kw)
+    lams = [0.0, 25.0, 400.0]
+    Ts = [1, 2, 33, 34] if case == "short" else [1999]
+    kind = gen.KIND_ADVERSARIAL if case == "adversarial" else gen.KIND_MIX
+    with magus.Context(device=0, platform=plat) as ctx:
+        for T in Ts:
+            N = 70
+            x = gen.gen_traces(gen.SEEDS[2], N, T, kind=kind)
+            out = ctx.offline_bound(torch.from_numpy(x).cuda(), lams, full_grid=full_grid)
+            torch.cuda.synchronize()
+            got = out.cpu().numpy()
+            for n in range(0, N, 3):
+                for j, lam in enumerate(lams):
+                    ref = oracle.offline_bound(x[:, n], lam, plat_o, full_grid=full_grid)
+                    assert np.array_equal(got[n, j], ref), (case, T, n, lam)
