@@ -143,7 +143,7 @@ typedef struct {
   uint64_t reserved;
 } magus_base;
 
-/* Per-config totals over traces: exact integer sums (uint64[16]) so that the
+/* Per-config totals over traces: exact integer sums (uint64[MAGUS_TOT_WORDS = 18]) so that the
  * cross-trace and cross-GPU reduction is order-free and bit-reproducible.
  * The q sums are split into 32-bit limbs (q = hi*2^32 + lo per trace) so that
  * each limb sum fits in 64 bits for any n_traces < 2^32, which also makes a

@@ -2,20 +2,24 @@
 // time-segmented replay of Alg. 1-3 + model M, in ONE launch per (W, H).
 //
 // Layout and mapping:
-//   * traces are time-major fp32 x[t][ld]; one CTA owns 128 consecutive
-//     traces x one time segment [t0, t1) x one config; one consumer thread
-//     owns one trace and scans it sequentially.
-//   * a producer warp streams [32 steps x 128 traces] boxes (16 KB) into a
-//     shared-memory ring with cp.async.bulk.tensor (TMA) completing on
-//     mbarriers.  For a compile-time W the Alg. 1 lag x[t-W+1] is kept in
-//     registers (each sample is widened to fp64 once), so a stage is released
-//     as soon as its word is done (3 stages, 4 CTAs/SM).
+//   * traces are time-major fp32 x[t][ld]; one CTA owns TR consecutive traces
+//     (512 for one config per thread -- one CTA per SM, 16 consumer warps on
+//     one ring; 128 for the config bundles of the sweeps, 3 CTAs per SM) x one
+//     time segment [t0, t1) x one bundle of configs; one consumer thread owns
+//     one trace and scans it sequentially.
+//   * a producer warp streams [32 steps x 128 traces] TMA boxes (16 KB each,
+//     TR / 128 per stage) into a shared-memory ring with
+//     cp.async.bulk.tensor completing on mbarriers.  For a compile-time W the
+//     Alg. 1 lag x[t-W+1] is kept in registers (each sample is widened to
+//     fp64 once), so a stage is released as soon as its word is done
+//     (3 stages).
 //   * each consumer handles 32 steps at a time ("a word"): per sample it only
 //     computes the Alg. 1 predicates (delta vs. host-inverted thresholds,
 //     precompute.cpp) and the stretch flag, packed into 32-bit masks.  Alg. 2
 //     (count of the H previous events >= k) is a bit-sliced carry-save
 //     counter over 32 positions at once; Alg. 3's sample-and-hold of the
-//     frequency is a 5-step log-depth forward fill; every counter is a popc.
+//     frequency is one carry-chain add (forward_fill); every counter is a
+//     popc.
 //   * segments are exact (DESIGN 6.3): p_t and hi_t depend only on
 //     x[t-W-H+1..t], so a segment re-reads a halo of ceil((W+H-1)/32) words;
 //     the only carried state is dec[t0-1].  A segment scans under a
