@@ -315,8 +315,8 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   extern __shared__ __align__(1024) float sm[];
   __shared__ __align__(8) uint64_t full_bar[kStages];
   __shared__ __align__(8) uint64_t empty_bar[kStages];
-  __shared__ uint32_t sh_last, sh_last2;
-  __shared__ int32_t sh_work[3];  // segment, bundle, group of this CTA
+  __shared__ uint32_t sh_last;
+  __shared__ int32_t sh_work[4];  // segment, bundle, group of this CTA; its ticket
   __shared__ unsigned long long sh_red[kConsumerWarps][kTotAcc];
   // digest multiplier of each staged word, delivered by a 16-B bulk copy from
   // the context's table on the stage's own full barrier (async proxy, like
@@ -333,6 +333,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
     // tickets, so they start together and stream the same trace tiles while
     // those are still in L2
     const uint32_t ticket = atomicAdd(wk.ticket, 1u);
+    sh_work[3] = (int32_t)ticket;
     const uint32_t per_seg = (uint32_t)ngroups * (uint32_t)nbund;
     const uint32_t sg = ticket / per_seg, rem = ticket - sg * per_seg;
     sh_work[0] = (int32_t)sg;
@@ -349,6 +350,24 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   }
   __syncthreads();
+  if (sh_work[3] == 0 && wk.totals) {
+    // The first CTA of the launch initialises the totals rows of the launch's
+    // configs (the finalisers add into them, so no per-group hand-off through
+    // a second arrival counter is needed) and raises the launch's flag.
+    const int32_t rows = nbund * NB;
+    for (int i = threadIdx.x; i < rows * MAGUS_TOT_WORDS; i += blockDim.x) {
+      const int32_t c = bundles[i / MAGUS_TOT_WORDS];
+      const int w = i % MAGUS_TOT_WORDS;
+      if (c >= 0)
+        wk.totals[(int64_t)c * MAGUS_TOT_WORDS + w] =
+            w == MAGUS_TOT_N_TRACES ? (uint64_t)N : (w == MAGUS_TOT_N_STEPS ? (uint64_t)N * (uint64_t)T : 0ull);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      st_release(wk.ticket + kTotalsFlagWord, 1u);
+    }
+  }
 
   const int32_t s = sh_work[0];
   const int32_t bidx = sh_work[1];
@@ -844,31 +863,16 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
           if (lane == 0) sh_red[warp][q] = v;
         }
         consumer_sync<TR>();
-        if (tid < kTotAcc) {
+        if (tid < kTotAcc) {  // accumulators 0..12 -> words 1..13; 13, 14 -> bursts (exact integer adds)
           unsigned long long v = 0;
           for (int q = 0; q < kConsumerWarps; ++q) v += sh_red[q][tid];
-          atomicAdd(wk.tacc + (int64_t)c * kTotAcc + tid, v);
+          // the launch's first CTA initialised the rows (its flag, normally
+          // raised long before any group is complete)
+          while (ld_acquire(wk.ticket + kTotalsFlagWord) == 0u) __nanosleep(MAGUS_LOOKBACK_SLEEP);
+          const int word = tid < 13 ? 1 + tid : MAGUS_TOT_BURST_BASE + (tid - 13);
+          atomicAdd(reinterpret_cast<unsigned long long*>(wk.totals + (int64_t)c * MAGUS_TOT_WORDS + word), v);
         }
-        __threadfence();
-        consumer_sync<TR>();
-        if (tid == 0) sh_last2 = (atomicAdd(wk.tarrive + c, 1u) == (uint32_t)(ngroups - 1));
-        consumer_sync<TR>();
-        if (sh_last2) {
-          __threadfence();
-          uint64_t* out = wk.totals + (int64_t)c * MAGUS_TOT_WORDS;
-          if (tid < kTotAcc) {  // accumulators 0..12 -> words 1..13; 13, 14 -> bursts
-            const int word = tid < 13 ? 1 + tid : MAGUS_TOT_BURST_BASE + (tid - 13);
-            out[word] = __ldcg(wk.tacc + (int64_t)c * kTotAcc + tid);
-            wk.tacc[(int64_t)c * kTotAcc + tid] = 0ULL;
-          }
-          if (tid == 0) {
-            out[MAGUS_TOT_N_TRACES] = (uint64_t)N;
-            out[MAGUS_TOT_N_STEPS] = (uint64_t)N * (uint64_t)T;
-            out[MAGUS_TOT_RESERVED] = 0;
-            wk.tarrive[c] = 0;
-          }
-        }
-        consumer_sync<TR>();  // sh_red / sh_last2 are reused by the next config
+        consumer_sync<TR>();  // sh_red is reused by the next config
       }
     }
     if (tid == 0) wk.arrive[(int64_t)c0 * ngroups + g] = 0;
@@ -885,6 +889,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
     if (atomicAdd(wk.done, 1u) == gridDim.x - 1) {
       *wk.ticket = 0;
       *wk.done = 0;
+      wk.ticket[kTotalsFlagWord] = 0;
     }
   }
 }

@@ -59,8 +59,8 @@ struct StreamWork {
   uint32_t* status;              // [C][nseg][N] epoch<<3 | last_min<<2 | seen<<1 | 1
   unsigned long long* acc;       // [C][kAccFields][N] segment sums
   uint32_t* arrive;              // [C][ngroups] finished segments
-  unsigned long long* tacc;      // [C][kTotAccWords] totals under construction
-  uint32_t* tarrive;             // [C] finished groups
+  unsigned long long* tacc;      // (unused since the finalisers add into the totals rows)
+  uint32_t* tarrive;             // (unused)
   uint32_t epoch;
   magus_summary* summary;        // [C][N] or NULL
   magus_base* base;              // [N] or NULL
@@ -82,6 +82,9 @@ struct StreamWork {
 // right after the ticket words (ticket[2..3] as a u64, NULL = off), so the
 // kernel's parameter block -- and its register allocation -- is unchanged.
 constexpr int kTraceSlotWords = 2;
+// ticket[4]: raised (1) once the launch's first CTA has initialised the
+// totals rows; cleared with the ticket by the launch's last CTA
+constexpr int kTotalsFlagWord = 4;
 // resume state layout: acc [C][kAccFields][N] u64, then carry [C][N] u32
 inline size_t resume_state_bytes(int64_t N, int32_t C) {
   return 8 * (size_t)kAccFields * (size_t)C * (size_t)N + 4 * (size_t)C * (size_t)N;
