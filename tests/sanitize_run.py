@@ -4,7 +4,7 @@ synccheck / initcheck) runs of the TMA + mbarrier + look-back kernels.
   compute-sanitizer --tool racecheck python tests/sanitize_run.py
 
 Exercises: several segments (look-back), a ragged trace group and tail word,
-bundles (NB = 4), bursts, decisions output, the per-sample kernel, the
+bundles (NB = 4, 128-trace CTAs), one config (the 512-trace CTA), bursts, decisions output, the per-sample kernel, the
 sequential / speculative / walk kernels (level output) and the DP.
 Exits non-zero if the results disagree with the oracle.
 """
@@ -35,15 +35,21 @@ def main():
     ref = oracle.replay(x, po, oracle.platform(burst=12000.0), want_dec=True)
     ok = True
     with magus.Context(device=0, platform=plat) as ctx:
-        for kernel, segs in ((magus.KERNEL_STREAM, 5), (magus.KERNEL_REFERENCE, 0)):
+        # the bundles (128-trace CTAs), one config (the 512-trace CTA, its
+        # totals initialised by the launch's first CTA), the per-sample kernel
+        for kernel, segs, sub in ((magus.KERNEL_STREAM, 5, [0, 1, 2, 3]), (magus.KERNEL_STREAM, 5, [2]),
+                                  (magus.KERNEL_REFERENCE, 0, [0, 1, 2, 3])):
             ctx.set_option(magus.OPT_KERNEL, kernel)
             ctx.set_option(magus.OPT_SEGMENTS, segs)
-            r = ctx.replay(xd, pols, n_traces=N, want_decisions=True)
+            r = ctx.replay(xd, [pols[i] for i in sub], n_traces=N, want_decisions=True)
             torch.cuda.synchronize()
             got = r.summary_numpy()
-            ok &= bool(np.array_equal(got["energy_j"], ref.summary["energy"]))
-            ok &= bool(np.array_equal(got["digest"], ref.summary["digest"]))
-            ok &= bool(np.array_equal(r.decisions_numpy().transpose(0, 2, 1), oracle.decision_words(ref.dec, 8)))
+            ok &= bool(np.array_equal(got["energy_j"], ref.summary["energy"][sub]))
+            ok &= bool(np.array_equal(got["digest"], ref.summary["digest"][sub]))
+            ok &= bool(np.array_equal(r.decisions_numpy().transpose(0, 2, 1), oracle.decision_words(ref.dec[sub], 8)))
+            for j, i in enumerate(sub):
+                ok &= bool(np.array_equal(r.totals_numpy()[j], oracle.totals(ref.summary[i], ref.base, T,
+                                                                             oracle.platform(burst=12000.0))[0]))
         # the sequential (f3), speculative (f3, every guess wrong at warm-up
         # 1) and walk (f4, several segments) kernels, with level output
         vpols = [magus.make_policy(variant=1), magus.make_policy(variant=2, step=2),
@@ -68,9 +74,11 @@ def main():
             ok &= bool(np.array_equal(rr.summary_numpy()["energy_j"], vref.summary["energy"][idx]))
         ctx.set_option(magus.OPT_KERNEL, magus.KERNEL_AUTO)
         ctx.set_option(magus.OPT_SEGMENTS, 0)
-        out = ctx.offline_bound(xd[:200, :8], [0.0, 100.0])
-        torch.cuda.synchronize()
-        ok &= bool(np.array_equal(out.cpu().numpy()[3, 1], oracle.offline_bound(x[:200, 3], 100.0)))
+        for full in (False, True):  # f2: the scalar-path binary kernel, the two-lane grid kernel
+            out = ctx.offline_bound(xd[:200, :8], [0.0, 100.0], full_grid=full)
+            torch.cuda.synchronize()
+            ok &= bool(np.array_equal(out.cpu().numpy()[3, 1],
+                                      oracle.offline_bound(x[:200, 3], 100.0, full_grid=full)))
     print("sanitize workload parity:", "ok" if ok else "MISMATCH")
     return 0 if ok else 1
 
