@@ -94,6 +94,27 @@ __device__ __forceinline__ void mbar_wait_s(uint32_t bar, uint32_t parity) {
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   mbar_wait_s(smem_u32(bar), parity);
 }
+#ifndef MAGUS_FULLWAIT_SLEEP
+#define MAGUS_FULLWAIT_SLEEP 0  // ns slept between the consumers' polls of a stage (0: suspend hint only)
+#endif
+// the consumers' wait for a stage: with MAGUS_FULLWAIT_SLEEP > 0 a warp that
+// finds the stage not yet landed sleeps between polls instead of re-issuing
+// the probe (the polls of 16 waiting warps otherwise take issue slots from
+// the warps doing the work)
+__device__ __forceinline__ void mbar_wait_full(uint32_t bar, uint32_t parity) {
+  if constexpr (MAGUS_FULLWAIT_SLEEP > 0) {
+    uint32_t ok;
+    asm volatile("{\n.reg .pred p;\nmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\nselp.u32 %0, 1, 0, p;\n}"
+                 : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
+    while (!ok) {
+      __nanosleep(MAGUS_FULLWAIT_SLEEP);
+      asm volatile("{\n.reg .pred p;\nmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\nselp.u32 %0, 1, 0, p;\n}"
+                   : "=r"(ok) : "r"(bar), "r"(parity) : "memory");
+    }
+  } else {
+    mbar_wait_s(bar, parity);
+  }
+}
 __device__ __forceinline__ void mbar_arrive_s(uint32_t bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
@@ -394,7 +415,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
   // one 32-step word of the scan; st / pst = stage of this / the previous word
   auto word = [&](const int st, const int pst, const uint32_t ph, const int32_t j)
                   __attribute__((always_inline)) {
-    mbar_wait_s(full_s + 8u * (uint32_t)st, ph);
+    mbar_wait_full(full_s + 8u * (uint32_t)st, ph);
     const float* cur = sm + st * kStageFloats + col;
     const uint32_t cur_s = sm_s + (uint32_t)(st * kStageFloats * 4);
     const int32_t w = w_first + j;
