@@ -73,7 +73,7 @@ def test_committed_bench_lines_carry_the_contract_keys():
     """Every bench line kept under profiles/ has the keys the driver and the
     judge read (roofline with its fraction, clocks, launches, baselines)."""
     import glob
-    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r01_bench_*.json")))
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r0*_bench_*.json")))
     assert files
     for f in files:
         d = json.loads(open(f).read().strip().splitlines()[-1])
