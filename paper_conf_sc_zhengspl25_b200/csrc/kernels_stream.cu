@@ -39,6 +39,11 @@
 #include "bitops.cuh"
 #include "device_common.cuh"
 
+#ifndef MAGUS_BUNDLE_OCC
+#define MAGUS_BUNDLE_OCC 4  // CTAs per SM of the compile-time-W config-bundle kernels (NB > 1): with
+                            // 2 stages of 16 KB and <= 102 registers, 4 fit (config 3: 25.3 -> 24.0 ms
+                            // against 3 CTAs x 3 stages; 4 CTAs x 3 stages do not fit the shared memory)
+#endif
 #ifndef MAGUS_LOOKBACK_SLEEP
 #define MAGUS_LOOKBACK_SLEEP 32  // ns between polls of a predecessor's segment status
 #endif
@@ -188,13 +193,13 @@ template <int W_T, int TR>
 struct Stages {
   // register lag (compile-time W): a stage is free once its word is read;
   // runtime W reads the lag from the previous stage, held one word longer.
-  static constexpr int n = W_T > 0 ? 3 : 4;
+  static constexpr int n = W_T > 0 ? (TR == 128 && MAGUS_BUNDLE_OCC > 3 ? 2 : 3) : 4;
   static constexpr int smem = n * Cta<TR>::stage_floats * 4;
 };
 // CTAs per SM the launch bounds aim for: NB configs per thread cost registers
 template <int W_T, int NB, int TR>
 struct Occ {
-  static constexpr int v = TR > 128 ? 1 : (NB == 1 ? (W_T > 0 ? 4 : 3) : 3);
+  static constexpr int v = TR > 128 ? 1 : (NB == 1 ? (W_T > 0 ? 4 : 3) : (W_T > 0 ? MAGUS_BUNDLE_OCC : 3));
 };
 
 // Per-config state of a bundle (NB configs that share W, H, L, tau_inc and
