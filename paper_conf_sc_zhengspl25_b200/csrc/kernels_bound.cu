@@ -507,7 +507,7 @@ constexpr int kBinChunk = 32;  // steps per staged chunk
 __global__ void __launch_bounds__(32)
 bound_binary_free_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
                          const double* __restrict__ lambdas, int32_t nl, DevPlatform plat, double bw_max,
-                         double p_lo, double p_span, float xthr0, double* __restrict__ out) {
+                         double p_lo, double p_span, float xthr0, float xthr_max, double* __restrict__ out) {
   __shared__ float s_x[2][kBinChunk][32];
   const int lane = threadIdx.x;
   const int64_t gid = (int64_t)blockIdx.x * 32 + lane;
@@ -578,25 +578,38 @@ bound_binary_free_kernel(const float* __restrict__ x, int64_t N, int64_t T, int6
       // chunk's start for the careful sweep below
       const double m1s = m1, E1s = E1, T1s = T1;
       bool tie = false;
+      // branch-free steps (so consecutive steps overlap): the r_min level's
+      // model-M cost is computed for every sample (q = 0 below its capacity
+      // gives exactly the q = 0 constants), the r_max level's only in chunks
+      // where some lane's sample exceeds even that capacity (warp-uniform)
+      bool over_max = false;
+#pragma unroll 8
+      for (int k = 0; k < kn; ++k) over_max |= xs[k * 32] > xthr_max;
+      if (__any_sync(0xFFFFFFFFu, over_max)) {
 #pragma unroll 4
-      for (int k = 0; k < kn; ++k) {
-        const float xf = xs[k * 32];
-        if (__any_sync(0xFFFFFFFFu, xf > xthr0)) {  // some lane has a stretch
+        for (int k = 0; k < kn; ++k) {
           double c0, c1, e0, e1, tau0, tau1;
-          costs(xf, c0, c1, e0, e1, tau0, tau1);
+          costs(xs[k * 32], c0, c1, e0, e1, tau0, tau1);
           const double s0 = m1 + c0, s1 = m1 + c1;
           tie |= s0 == s1;
           const bool up = s1 < s0;
           m1 = up ? s1 : s0;
           E1 = E1 + (up ? e1 : e0);
           T1 = T1 + (up ? tau1 : tau0);
-        } else {
-          const double s0 = m1 + cf0, s1 = m1 + cf1;
+        }
+      } else {
+#pragma unroll 8
+        for (int k = 0; k < kn; ++k) {
+          const double xd = (double)xs[k * 32];
+          const double tau0 = dt + cQ * q_as_double(xd, invB0);
+          const double e0 = P0 * tau0;
+          const double c0 = e0 + lam * tau0;
+          const double s0 = m1 + c0, s1 = m1 + cf1;
           tie |= s0 == s1;
           const bool up = s1 < s0;
           m1 = up ? s1 : s0;
-          E1 = E1 + (up ? Pdt1 : Pdt0);
-          T1 = T1 + dt;
+          E1 = E1 + (up ? Pdt1 : e0);
+          T1 = T1 + (up ? dt : tau0);
         }
       }
       if (__any_sync(0xFFFFFFFFu, tie)) {
@@ -662,7 +675,7 @@ int launch_bound(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t l
   const unsigned warps = (unsigned)((N * nl + 15) / 16);  // 16 chains (2 lanes each) per warp
   if (L == 2 && plat.e_sw == 0.0 && plat.t_sw == 0.0)
     bound_binary_free_kernel<<<(unsigned)((N * nl + 31) / 32), 32, 0, s>>>(x, N, T, ld, lambdas_dev, nl, plat,
-                                                                         bw_max, p_lo, p_span, thr.x[0], out);
+                                                                         bw_max, p_lo, p_span, thr.x[0], thr.x[1], out);
   else if (L == 2)  // two levels with switch costs: the branch-free per-step kernel
     bound_binary_kernel<<<blocks, kBoundThreads, 0, s>>>(x, N, T, ld, lambdas_dev, nl, plat, bw_max, p_lo,
                                                          p_span, out);
