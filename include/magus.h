@@ -433,9 +433,16 @@ enum {
                                  1024)); any value gives the same results   */
   MAGUS_OPT_TRACE = 6,        /* 1: the stream kernel records a per-CTA
                                  timeline (diagnostics; magus_get_trace)     */
-  MAGUS_OPT_NARROW = 7        /* 1: the stream kernel's one-config path uses
+  MAGUS_OPT_NARROW = 7,       /* 1: the stream kernel's one-config path uses
                                  128-trace CTAs (4 per SM) instead of the
                                  default 512-trace CTA per SM (A/B option;
+                                 results are identical)                      */
+  MAGUS_OPT_FAMILY = 8        /* 0 (default): a (W, H) group of <= 16 bundles
+                                 of 4 configs with <= 8 distinct tau_inc and
+                                 tau_dec thresholds (a sweep grid, Sec. 6.4)
+                                 runs on the family kernel, which compares
+                                 each sample once for the whole group; 1: the
+                                 per-bundle stream kernel (A/B option;
                                  results are identical)                      */
 };
 magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value);

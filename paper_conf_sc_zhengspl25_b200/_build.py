@@ -15,7 +15,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 BUILD = os.path.join(HERE, "build")
 LIB = os.path.join(HERE, "libmagus.so")
-SOURCES = ["api.cu", "precompute.cpp", "kernels_ref.cu", "kernels_seq.cu", "kernels_walk.cu", "kernels_spec.cu", "kernels_stream.cu", "kernels_post.cu",
+SOURCES = ["api.cu", "precompute.cpp", "kernels_ref.cu", "kernels_seq.cu", "kernels_walk.cu", "kernels_spec.cu", "kernels_stream.cu", "kernels_family.cu", "kernels_post.cu",
            "kernels_bound.cu", "comm.cpp"]
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

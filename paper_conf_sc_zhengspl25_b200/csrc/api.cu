@@ -26,6 +26,7 @@ struct magus_ctx_s {
   int sms = 148;
   // options
   int64_t opt_kernel = 0, opt_segments = 0, opt_timing = 0, opt_waves = 0, opt_trace = 0, opt_narrow = 0;
+  int64_t opt_family = 0;  // 0: family kernel for the groups it takes; 1: bundle kernels only
   void* trace_dev = nullptr;   // MAGUS_OPT_TRACE timeline [trace_cap][8]
   int64_t trace_cap = 0, trace_n = 0;
   bool trace_armed = false;          // scratch holds a timeline address
@@ -48,6 +49,8 @@ struct magus_ctx_s {
     int32_t W, H, NB;   // kernel specialisation
     int64_t off;        // first bundle (rows of NB config indices) in the device table
     int32_t nbund;
+    bool fam_ok;        // the family kernel can take the whole group (kernels_family.cu)
+    FamilyDev fam;
   };
   std::vector<LaunchGroup> groups;  // one stream launch each
   int64_t opt_bundle = 0;           // 0 auto, else force NB in {1, 2, 4}
@@ -169,13 +172,36 @@ magus_status upload_policies(magus_ctx ctx, const magus_policy* params, int32_t 
     size_t maxsz = 1;
     for (auto& b : wh.second) maxsz = std::max(maxsz, b.second.size());
     int32_t NB = ctx->opt_bundle ? (int32_t)ctx->opt_bundle : (maxsz >= 3 ? 4 : (int32_t)maxsz);
-    magus_ctx_s::LaunchGroup lg{wh.first.first, wh.first.second, NB, 0, 0};
+    magus_ctx_s::LaunchGroup lg{wh.first.first, wh.first.second, NB, 0, 0, false, {}};
     lg.off = (int64_t)table.size();
+    // family: the distinct inverted thresholds of the group's bundles
+    std::vector<uint64_t> dinc, ddec;
+    std::vector<uint8_t> bi, bd;
     for (auto& b : wh.second) {
       const auto& v = b.second;
+      auto idx = [](std::vector<uint64_t>& tab, uint64_t key) {
+        for (size_t i = 0; i < tab.size(); ++i)
+          if (tab[i] == key) return (uint8_t)i;
+        tab.push_back(key);
+        return (uint8_t)(tab.size() - 1);
+      };
+      const uint8_t ii = idx(dinc, b.first.first), id = idx(ddec, b.first.second);
       for (size_t i = 0; i < v.size(); i += (size_t)NB) {
         for (int32_t k = 0; k < NB; ++k) table.push_back(i + k < v.size() ? v[i + k] : -1);
         lg.nbund++;
+        bi.push_back(ii);
+        bd.push_back(id);
+      }
+    }
+    lg.fam_ok = family_supported(lg.W, lg.H, NB, lg.nbund, (int32_t)dinc.size(), (int32_t)ddec.size());
+    if (lg.fam_ok) {
+      lg.fam.ni = (int32_t)dinc.size();
+      lg.fam.nd = (int32_t)ddec.size();
+      for (size_t i = 0; i < dinc.size(); ++i) std::memcpy(&lg.fam.d_inc[i], &dinc[i], 8);
+      for (size_t i = 0; i < ddec.size(); ++i) std::memcpy(&lg.fam.d_dec[i], &ddec[i], 8);
+      for (int32_t b = 0; b < lg.nbund; ++b) {
+        lg.fam.bi[b] = bi[(size_t)b];
+        lg.fam.bd[b] = bd[(size_t)b];
       }
     }
     ctx->groups.push_back(lg);
@@ -228,8 +254,28 @@ int64_t stream_groups(magus_ctx ctx, int64_t N, int W, int H, int NB) {  // CTAs
   return (N + tr - 1) / tr;
 }
 
+// the family kernel takes the group: every bundle in one CTA (no burst counters there)
+bool use_family(magus_ctx ctx, const magus_ctx_s::LaunchGroup& g) {
+  return g.fam_ok && ctx->opt_family == 0 && ctx->dplat.burst_on == 0;
+}
+int64_t group_ctas(magus_ctx ctx, int64_t N, const magus_ctx_s::LaunchGroup& g, int64_t nseg) {
+  if (use_family(ctx, g)) return (N + family_cta_traces() - 1) / family_cta_traces() * nseg;
+  return stream_groups(ctx, N, g.W, g.H, g.NB) * g.nbund * nseg;
+}
+int group_ctas_per_sm(magus_ctx ctx, const magus_ctx_s::LaunchGroup& g) {
+  if (use_family(ctx, g)) {
+    auto key = std::make_pair(-1 - g.nbund, g.H == 10 ? 10 : 0);
+    auto it = ctx->ctas_cache.find(key);
+    if (it != ctx->ctas_cache.end()) return it->second;
+    const int v = family_ctas_per_sm(g.H, g.nbund);
+    ctx->ctas_cache[key] = v;
+    return v;
+  }
+  return ctas_per_sm(ctx, g.W, g.H, g.NB);
+}
+
 magus_status encode_tmap(magus_ctx ctx, CUtensorMap* map, const float* x, int64_t N, int64_t T,
-                         int64_t ld) {
+                         int64_t ld, uint32_t box_traces = 128) {
   if (!ctx->encode) {
     void* fn = nullptr;
     cudaDriverEntryPointQueryResult q;
@@ -240,7 +286,7 @@ magus_status encode_tmap(magus_ctx ctx, CUtensorMap* map, const float* x, int64_
   }
   cuuint64_t dims[2] = {(cuuint64_t)N, (cuuint64_t)T};
   cuuint64_t strides[1] = {(cuuint64_t)ld * 4};
-  cuuint32_t box[2] = {128, 32};
+  cuuint32_t box[2] = {box_traces, 32};
   cuuint32_t estr[2] = {1, 1};
   CUresult r = ctx->encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)x, dims, strides, box,
                            estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
@@ -522,6 +568,9 @@ magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value) {
     case MAGUS_OPT_NARROW:
       ctx->opt_narrow = value ? 1 : 0;
       return MAGUS_OK;
+    case MAGUS_OPT_FAMILY:
+      ctx->opt_family = value ? 1 : 0;
+      return MAGUS_OK;
     case MAGUS_OPT_WAVES:
       if (value < 0 || value > 64) return fail(ctx, MAGUS_ERR_INVALID_ARG, "waves not in [0, 64]");
       ctx->opt_waves = value;
@@ -618,8 +667,8 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
         if ((Tr + len - 1) / len != cand) continue;  // not realisable with 32-step segments
         double cost = 0.0;
         for (auto& g : ctx->groups) {
-          const int64_t slots = (int64_t)ctx->sms * std::max(1, ctas_per_sm(ctx, g.W, g.H, g.NB));
-          const int64_t ctas = stream_groups(ctx, N, g.W, g.H, g.NB) * g.nbund * cand;
+          const int64_t slots = (int64_t)ctx->sms * std::max(1, group_ctas_per_sm(ctx, g));
+          const int64_t ctas = group_ctas(ctx, N, g, cand);
           const int64_t halo = cand > 1 ? ((g.W + g.H - 1 + 31) / 32) * 32 : 0;
           cost += (double)((ctas + slots - 1) / slots) * (double)(len + halo + 96);
         }
@@ -632,7 +681,7 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
       int per_sm = 1 << 30;
       int64_t nbund = 0;
       for (auto& g : ctx->groups) {
-        per_sm = std::min(per_sm, ctas_per_sm(ctx, g.W, g.H, g.NB));
+        per_sm = std::min(per_sm, group_ctas_per_sm(ctx, g));
         nbund += g.nbund;
       }
       if (per_sm < 1) per_sm = 1;
@@ -770,7 +819,7 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     // scratch of the fused kernel: counters + accumulators (zero, self-cleaning)
     // followed by the epoch-tagged segment status words
     const size_t off_arrive = 256;
-    const size_t off_tarrive = off_arrive + align_up(4 * (size_t)(C * ngroups), 256);
+    const size_t off_tarrive = off_arrive + align_up(4 * (size_t)(C * ((N + 31) / 32)), 256);  // any CTA width
     const size_t off_tacc = off_tarrive + align_up(4 * (size_t)C, 256);
     const size_t off_acc = off_tacc + align_up(8 * kTotAccWords * (size_t)C, 256);
     const size_t off_status = off_acc + align_up(8 * (size_t)kAccFields * (size_t)(C * N), 256);
@@ -812,7 +861,7 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
       void* tp = nullptr;
       if (ctx->opt_trace) {
         int64_t grid_all = 0;
-        for (auto& g : ctx->groups) grid_all += stream_groups(ctx, N, g.W, g.H, g.NB) * nseg * g.nbund;
+        for (auto& g : ctx->groups) grid_all += group_ctas(ctx, N, g, nseg);
         if (grid_all > ctx->trace_cap) {
           CK(cudaStreamSynchronize(ctx->stream));
           if (ctx->trace_dev) cudaFree(ctx->trace_dev);
@@ -847,9 +896,15 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
       ctx->mul_nw = cap;
     }
     wk.mul = (const unsigned long long*)ctx->mul_dev;
-    CUtensorMap map, map_mul;
+    CUtensorMap map, map_mul, map32;
     st = encode_tmap(ctx, &map, traces, N, T, ld);
     if (st != MAGUS_OK) return st;
+    bool any_family = false;
+    for (auto& g : ctx->groups) any_family = any_family || use_family(ctx, g);
+    if (any_family) {
+      st = encode_tmap(ctx, &map32, traces, N, T, ld, (uint32_t)family_cta_traces());
+      if (st != MAGUS_OK) return st;
+    }
     st = encode_mul_tmap(ctx, &map_mul);
     if (st != MAGUS_OK) return st;
     if (ctx->opt_timing) CK(cudaEventRecord(ev0, ctx->stream));
@@ -857,8 +912,11 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     for (size_t gi = 0; gi < ctx->groups.size(); ++gi) {
       auto& g = ctx->groups[gi];
       int grid = 0;
-      int r = launch_stream(ctx->stream, &map, &map_mul, N, tb + T, dev_policies(ctx), dev_cidx(ctx, g.off), g.nbund,
-                            g.NB, g.W, g.H, ctx->dplat, nseg, seg_len, wk, ctx->opt_narrow != 0, &grid);
+      int r = use_family(ctx, g)
+                  ? launch_family(ctx->stream, &map32, &map_mul, N, tb + T, dev_policies(ctx), dev_cidx(ctx, g.off),
+                                  g.nbund, g.H, g.fam, ctx->dplat, nseg, seg_len, wk, &grid)
+                  : launch_stream(ctx->stream, &map, &map_mul, N, tb + T, dev_policies(ctx), dev_cidx(ctx, g.off),
+                                  g.nbund, g.NB, g.W, g.H, ctx->dplat, nseg, seg_len, wk, ctx->opt_narrow != 0, &grid);
       if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "stream kernel launch");
       launched += r;
       grid_total += grid;

@@ -145,6 +145,25 @@ int nccl_comm_init(void** comm, const void* id_bytes, int nranks, int rank);
 int nccl_comm_destroy(void* comm);
 int nccl_allreduce_u64_sum(void* comm, uint64_t* buf, size_t count, cudaStream_t s);
 
+// Configuration-family kernel (kernels_family.cu): one CTA = 32 traces x one
+// time segment x every bundle of a (W, H) launch group (<= 16 bundles of 4
+// configs), the per-sample Alg. 1 compares done once for all of them against
+// the family's distinct inverted thresholds.
+constexpr int kFamMaxThr = 8;   // distinct d_inc / d_dec values of a family
+constexpr int kFamMaxBund = 16;
+struct FamilyDev {
+  double d_inc[kFamMaxThr], d_dec[kFamMaxThr];
+  int32_t ni, nd;
+  uint8_t bi[kFamMaxBund], bd[kFamMaxBund];  // bundle -> threshold indices
+};
+bool family_supported(int32_t W, int32_t H, int32_t NB, int32_t nbund, int32_t ni, int32_t nd);
+int family_cta_traces();
+int family_ctas_per_sm(int32_t H, int32_t nbund);
+int launch_family(cudaStream_t s, const void* tmap32 /* CUtensorMap, box 32 x 32 */, const void* tmap_mul,
+                  int64_t N, int64_t T, const DevPolicy* pol_dev, const int32_t* bundles_dev, int32_t nbund,
+                  int32_t H, const FamilyDev& fam, const DevPlatform& plat, int64_t nseg, int64_t seg_len,
+                  const StreamWork& wk, int* grid_out);
+
 bool stream_supported(int32_t W, int32_t H);
 // Fused stream kernel over nbund bundles of NB configs (bundles_dev:
 // [nbund][NB] global config indices, -1 = padding).  All configs of a launch
