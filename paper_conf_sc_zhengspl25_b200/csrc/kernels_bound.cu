@@ -590,10 +590,12 @@ bound_binary_free_kernel(const float* __restrict__ x, int64_t N, int64_t T, int6
         for (int k = 0; k < kn; ++k) {
           double c0, c1, e0, e1, tau0, tau1;
           costs(xs[k * 32], c0, c1, e0, e1, tau0, tau1);
-          const double s0 = m1 + c0, s1 = m1 + c1;
-          tie |= s0 == s1;
-          const bool up = s1 < s0;
-          m1 = up ? s1 : s0;
+          // without a tie, RN(m1 + c1) < RN(m1 + c0) <=> c1 < c0 (RN is
+          // monotone): the step's choice does not depend on m1, and the
+          // dependent chain is one add (the tie test runs beside it)
+          const bool up = c1 < c0;
+          tie |= (m1 + c0) == (m1 + c1);
+          m1 = m1 + (up ? c1 : c0);
           E1 = E1 + (up ? e1 : e0);
           T1 = T1 + (up ? tau1 : tau0);
         }
@@ -604,10 +606,9 @@ bound_binary_free_kernel(const float* __restrict__ x, int64_t N, int64_t T, int6
           const double tau0 = dt + cQ * q_as_double(xd, invB0);
           const double e0 = P0 * tau0;
           const double c0 = e0 + lam * tau0;
-          const double s0 = m1 + c0, s1 = m1 + cf1;
-          tie |= s0 == s1;
-          const bool up = s1 < s0;
-          m1 = up ? s1 : s0;
+          const bool up = cf1 < c0;
+          tie |= (m1 + c0) == (m1 + cf1);
+          m1 = m1 + (up ? cf1 : c0);
           E1 = E1 + (up ? Pdt1 : e0);
           T1 = T1 + (up ? dt : tau0);
         }
@@ -660,6 +661,184 @@ bound_binary_free_kernel(const float* __restrict__ x, int64_t N, int64_t T, int6
   o[2] = T1;
 }
 
+// ---------------------------------------------------------------------------
+// bound_binary_shared_kernel: bound_binary_free_kernel when nl divides 32 (a
+// warp holds 32 / nl whole traces, lanes = (trace slot, lambda)).  The
+// lambda-independent model-M terms of a step (tau, e = P tau of both levels)
+// are computed once per (trace, step) into shared memory by the whole warp
+// and read by the trace's nl lanes; samples are staged [step][trace slot]
+// (one copy per trace, not per lane).  A lane's step is then c = e + lam tau,
+// the choice (c1 < c0: no tie), the tie test and three adds.  Same fp64
+// operations as the free kernel (and the oracle DP), bit for bit.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void cp_async4z(float* dst, const float* src, bool valid) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"((uint32_t)__cvta_generic_to_shared(dst)),
+               "l"(src), "r"(valid ? 4 : 0)
+               : "memory");
+}
+
+__global__ void __launch_bounds__(32)
+bound_binary_shared_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
+                           const double* __restrict__ lambdas, int32_t nl, DevPlatform plat, double bw_max,
+                           double p_lo, double p_span, float xthr_max, double* __restrict__ out) {
+  __shared__ float s_x[2][kBinChunk][16];     // [buffer][step][trace slot]
+  __shared__ double2 s_te[kBinChunk][16][2];  // [step][trace slot][level] {tau, e}
+  const int lane = threadIdx.x;
+  const int lgnl = __ffs(nl) - 1, lgtpw = 5 - lgnl, tpw = 1 << lgtpw;
+  const int slot = lane >> lgnl, j = lane & (nl - 1);
+  const int64_t n0 = (int64_t)blockIdx.x * tpw;  // the warp's first trace
+  const int64_t n = n0 + slot;
+  const bool active = n < N;
+  const double lam = lambdas[j];
+  const int lmin = plat.r_min, lmax = plat.r_max;
+  const double invB0 = 1.0 / ((bw_max * (double)lmin) / (double)lmax);
+  const double invB1 = 1.0 / ((bw_max * (double)lmax) / (double)lmax);
+  const double P0 = p_lo + (p_span * (double)(lmin - lmin)) / (double)(lmax - lmin);
+  const double P1 = p_lo + (p_span * (double)(lmax - lmin)) / (double)(lmax - lmin);
+  const double dt = plat.dt, cQ = plat.cQ;
+  const double Pdt1 = P1 * dt;
+  const double cf1 = Pdt1 + lam * dt;  // e + lambda * tau at r_max, q = 0
+  double m1, E1, T1;
+  {
+    const double xd = (double)(active ? __ldg(x + n) : 0.0f);
+    const double tau1 = dt + cQ * q_as_double(xd, invB1);
+    const double e1 = P1 * tau1;
+    m1 = e1 + lam * tau1;
+    E1 = e1;
+    T1 = tau1;
+  }
+  bool general = false;
+  double V0 = 0.0, V1 = 0.0, E0 = 0.0, Ea = 0.0, T0 = 0.0, Ta = 0.0;
+  const int64_t nch = (T - 1 + kBinChunk - 1) / kBinChunk;
+  // a lane's (step, slot) items of a chunk: slot r_l, steps k_l + i * kstride
+  const int r_l = lane & (tpw - 1), k_l = lane >> lgtpw, kstride = 32 >> lgtpw;
+  const bool r_ok = n0 + r_l < N;
+  const float* xl = x + (r_ok ? n0 + r_l : 0);
+  const int64_t ldk = (int64_t)kstride * ld;
+  auto stage = [&](int64_t c) {
+    const int64_t t0 = 1 + c * kBinChunk;
+    const float* src = xl + (t0 + k_l) * ld;
+    float* dst = &s_x[c & 1][k_l][r_l];
+    int64_t t = t0 + k_l;
+    for (int i = 0; i < tpw; ++i) {
+      const bool ok = r_ok && t < T;
+      cp_async4z(dst, ok ? src : x, ok);
+      src += ldk;
+      dst += kstride * 16;
+      t += kstride;
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  if (nch > 0) stage(0);
+  for (int64_t c = 0; c < nch; ++c) {
+    if (c + 1 < nch) {
+      stage(c + 1);
+      asm volatile("cp.async.wait_group 1;" ::: "memory");
+    } else {
+      asm volatile("cp.async.wait_group 0;" ::: "memory");
+    }
+    __syncwarp();
+    const int64_t t0 = 1 + c * kBinChunk;
+    const int kn = (int)(T - t0 < kBinChunk ? T - t0 : kBinChunk);
+    auto costs = [&](float xf, double& c0, double& c1, double& e0, double& e1, double& tau0, double& tau1) {
+      const double xd = (double)xf;
+      tau0 = dt + cQ * q_as_double(xd, invB0);
+      tau1 = dt + cQ * q_as_double(xd, invB1);
+      e0 = P0 * tau0;
+      e1 = P1 * tau1;
+      c0 = e0 + lam * tau0;
+      c1 = e1 + lam * tau1;
+    };
+    bool redo = false;
+    if (!general) {
+      // the chunk's (tau, e) at r_min per (step, slot), once for the warp
+      bool over = false;
+      for (int k = k_l; k < kn; k += kstride) {
+        const float xf = s_x[c & 1][k][r_l];
+        const double tau0 = dt + cQ * q_as_double((double)xf, invB0);
+        s_te[k][r_l][0] = make_double2(tau0, P0 * tau0);
+        over |= xf > xthr_max;
+      }
+      const bool omax = __any_sync(0xFFFFFFFFu, over);
+      if (omax) {  // some sample exceeds even the capacity at r_max (rare): that level's terms too
+        for (int k = k_l; k < kn; k += kstride) {
+          const double tau1 = dt + cQ * q_as_double((double)s_x[c & 1][k][r_l], invB1);
+          s_te[k][r_l][1] = make_double2(tau1, P1 * tau1);
+        }
+      }
+      __syncwarp();
+      const double m1s = m1, E1s = E1, T1s = T1;
+      bool tie = false;
+      if (omax) {
+#pragma unroll 4
+        for (int k = 0; k < kn; ++k) {
+          const double2 a = s_te[k][slot][0], b = s_te[k][slot][1];
+          const double c0 = a.y + lam * a.x, c1 = b.y + lam * b.x;
+          const bool up = c1 < c0;  // without a tie <=> RN(m1 + c1) < RN(m1 + c0)
+          tie |= (m1 + c0) == (m1 + c1);
+          m1 = m1 + (up ? c1 : c0);
+          E1 = E1 + (up ? b.y : a.y);
+          T1 = T1 + (up ? b.x : a.x);
+        }
+      } else {
+#pragma unroll 8
+        for (int k = 0; k < kn; ++k) {
+          const double2 a = s_te[k][slot][0];
+          const double c0 = a.y + lam * a.x;
+          const bool up = cf1 < c0;
+          tie |= (m1 + c0) == (m1 + cf1);
+          m1 = m1 + (up ? cf1 : c0);
+          E1 = E1 + (up ? Pdt1 : a.y);
+          T1 = T1 + (up ? dt : a.x);
+        }
+      }
+      if (__any_sync(0xFFFFFFFFu, tie)) {
+        m1 = m1s; E1 = E1s; T1 = T1s;
+        redo = true;
+      }
+    }
+    if (general || redo) {
+#pragma unroll 1
+      for (int k = 0; k < kn; ++k) {
+        double c0, c1, e0, e1, tau0, tau1;
+        costs(s_x[c & 1][k][slot], c0, c1, e0, e1, tau0, tau1);
+        if (!general) {
+          const double s0 = m1 + c0, s1 = m1 + c1;
+          if (__any_sync(0xFFFFFFFFu, s0 == s1)) {
+            V0 = s0; V1 = s1;
+            E0 = E1 + e0; Ea = E1 + e1;
+            T0 = T1 + tau0; Ta = T1 + tau1;
+            general = true;
+          } else {
+            const bool up = s1 < s0;
+            m1 = up ? s1 : s0;
+            E1 = E1 + (up ? e1 : e0);
+            T1 = T1 + (up ? tau1 : tau0);
+          }
+        } else {
+          const bool st0 = V0 <= V1, st1 = V1 <= V0;
+          const double nV0 = (st0 ? V0 : V1) + c0, nE0 = (st0 ? E0 : Ea) + e0, nT0 = (st0 ? T0 : Ta) + tau0;
+          const double nV1 = (st1 ? V1 : V0) + c1, nE1 = (st1 ? Ea : E0) + e1, nT1 = (st1 ? Ta : T0) + tau1;
+          V0 = nV0; E0 = nE0; T0 = nT0;
+          V1 = nV1; Ea = nE1; Ta = nT1;
+        }
+      }
+    }
+    __syncwarp();  // s_x[c & 1] is restaged by chunk c + 2, s_te by the next chunk
+  }
+  if (general) {
+    const bool b1 = V1 < V0;
+    m1 = b1 ? V1 : V0;
+    E1 = b1 ? Ea : E0;
+    T1 = b1 ? Ta : T0;
+  }
+  if (!active) return;
+  double* o = out + (n * nl + j) * 3;
+  o[0] = m1;
+  o[1] = E1;
+  o[2] = T1;
+}
+
 int launch_bound(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,
                  const double* lambdas_dev, int32_t nl, bool full_grid, const DevPlatform& plat,
                  double bw_max, double p_lo, double p_span, double* out) {
@@ -673,7 +852,10 @@ int launch_bound(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t l
     thr.x[i] = i < L ? stretch_threshold(1.0 / ((bw_max * (double)l) / (double)plat.r_max)) : INFINITY;
   }
   const unsigned warps = (unsigned)((N * nl + 15) / 16);  // 16 chains (2 lanes each) per warp
-  if (L == 2 && plat.e_sw == 0.0 && plat.t_sw == 0.0)
+  if (L == 2 && plat.e_sw == 0.0 && plat.t_sw == 0.0 && nl >= 2 && 32 % nl == 0)
+    bound_binary_shared_kernel<<<(unsigned)((N + (32 / nl) - 1) / (32 / nl)), 32, 0, s>>>(
+        x, N, T, ld, lambdas_dev, nl, plat, bw_max, p_lo, p_span, thr.x[1], out);
+  else if (L == 2 && plat.e_sw == 0.0 && plat.t_sw == 0.0)
     bound_binary_free_kernel<<<(unsigned)((N * nl + 31) / 32), 32, 0, s>>>(x, N, T, ld, lambdas_dev, nl, plat,
                                                                          bw_max, p_lo, p_span, thr.x[0], thr.x[1], out);
   else if (L == 2)  // two levels with switch costs: the branch-free per-step kernel

@@ -123,7 +123,8 @@ def test_gpu_offline_bound_bit_exact(full_grid, r_max):
 @pytest.mark.gpu
 @pytest.mark.parametrize("full_grid", [False, True])
 @pytest.mark.parametrize("case", ["free_switch", "flat_power_ties", "tiny_switch", "adversarial", "short"])
-def test_gpu_offline_bound_modes_bit_exact(full_grid, case):
+@pytest.mark.parametrize("nl", [3, 8])
+def test_gpu_offline_bound_modes_bit_exact(full_grid, case, nl):
     """The throughput kernel's two bookkeeping modes: free
     switches (the paper's default: scalar path sums), equal power at every
     level (exact ties everywhere: per-level histories and the lowest-index
@@ -139,7 +140,9 @@ def test_gpu_offline_bound_modes_bit_exact(full_grid, case):
     plat.p_unc_min_w = kw.get("p_unc_min", plat.p_unc_min_w)
     plat.p_unc_max_w = kw.get("p_unc_max", plat.p_unc_max_w)
     plat_o = oracle.platform(**kw)
-    lams = [0.0, 25.0, 400.0]
+    # 8 lambdas: a warp holds whole traces (the binary kernel's shared
+    # per-(trace, step) model-M terms); 3: traces straddle warps
+    lams = [0.0, 25.0, 400.0] if nl == 3 else [0.0, 10.0, 25.0, 40.0, 160.0, 400.0, 2560.0, 1e6]
     Ts = [1, 2, 33, 34] if case == "short" else [1999]
     kind = gen.KIND_ADVERSARIAL if case == "adversarial" else gen.KIND_MIX
     with magus.Context(device=0, platform=plat) as ctx:
