@@ -839,6 +839,293 @@ bound_binary_shared_kernel(const float* __restrict__ x, int64_t N, int64_t T, in
   o[2] = T1;
 }
 
+// ---------------------------------------------------------------------------
+// bound_grid_free_kernel<L>: the full level grid with free switches (the
+// default platform) when nl divides 32.  As in the binary case, without a tie
+// every level's new value is m1 + c_l (a1 always stays, every other level
+// moves from it at no cost), so the state is (m1, E1, T1) and a step is
+// m1 += min_l c_l, E1 += e_a, T1 += tau_a (a = the argmin) -- valid while
+// RN(m1 + c_second) != RN(m1 + c_min) (monotone RN: then no other level ties
+// the minimum).  Levels at or above l*(x) (capacity >= x: q = 0) cost the
+// constants P_l dt + lam dt, increasing in l, so only cf_l* and cf_l*+1 can
+// be the minimum or runner-up among them; the levels below l* are stretched
+// (rare: ~4 % of the mix traces' samples exceed even the r_min capacity) and
+// their (tau, e) are computed in the lane.  l* per (trace, step) comes from
+// the warp's staged samples.  A tie anywhere in a chunk sends the warp back to
+// the chunk's start: the careful pass rebuilds every level's state at the
+// tie step (V_l = m1 + c_l, E_l = E1 + e_l, T_l = T1 + tau_l -- the oracle's
+// own sums, as no level tied before) and finishes with the oracle's
+// per-level recurrence.  Bit-identical to the oracle DP.
+// ---------------------------------------------------------------------------
+// shared loads by 32-bit window address (a generic pointer into a __shared__
+// array indexed at run time makes the compiler re-derive the window base --
+// an S2UR of the CTA id -- at every use)
+__device__ __forceinline__ double lds_f64a(uint32_t a) {
+  double v;
+  asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ float lds_f32a(uint32_t a) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ uint32_t lds_u8a(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+
+template <int L, int P>
+__global__ void __launch_bounds__(32)
+bound_grid_free_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_t ld,
+                       const double* __restrict__ lambdas, int32_t nl, int32_t lstep, DevPlatform plat,
+                       double bw_max, double p_lo, double p_span, const __grid_constant__ BoundThr thr,
+                       double* __restrict__ out) {
+  __shared__ float s_x[2][kBinChunk][16];       // [buffer][step][trace slot]
+  __shared__ __align__(16) uint8_t s_ls[kBinChunk][16];  // l* of (step, slot)
+  __shared__ double s_invB[L], s_P[L], s_Pdt[L];
+  __shared__ double s_V[L][32], s_E[L][32], s_T[L][32];  // per-level state after a tie (rare)
+  __shared__ float s_thr[32];
+  const int lane = threadIdx.x;
+  for (int i = lane; i < L; i += 32) {
+    const int l = plat.r_min + i * lstep;
+    const double B = (bw_max * (double)l) / (double)plat.r_max;
+    s_invB[i] = 1.0 / B;
+    s_P[i] = p_lo + (p_span * (double)(l - plat.r_min)) / (double)(plat.r_max - plat.r_min);
+    s_Pdt[i] = s_P[i] * plat.dt;
+  }
+  s_thr[lane] = lane < L ? thr.x[lane] : INFINITY;
+  __syncwarp();
+  const uint32_t a_x = (uint32_t)__cvta_generic_to_shared(&s_x[0][0][0]);
+  const uint32_t a_ls = (uint32_t)__cvta_generic_to_shared(&s_ls[0][0]);
+  const uint32_t a_invB = (uint32_t)__cvta_generic_to_shared(&s_invB[0]);
+  const uint32_t a_P = (uint32_t)__cvta_generic_to_shared(&s_P[0]);
+  const uint32_t a_Pdt = (uint32_t)__cvta_generic_to_shared(&s_Pdt[0]);
+  const uint32_t a_thr = (uint32_t)__cvta_generic_to_shared(&s_thr[0]);
+  // P lanes per chain (h = lane % P): they split the stretched levels of a
+  // slow step (l = h mod P) and merge by shuffles; 32 / P chains per warp
+  constexpr int kLgP = P == 1 ? 0 : (P == 2 ? 1 : (P == 4 ? 2 : 3));
+  const int h = lane & (P - 1), ch = lane >> kLgP;
+  const int lgnl = __ffs(nl) - 1, lgtpw = 5 - kLgP - lgnl, tpw = 1 << lgtpw;
+  const int slot = ch >> lgnl, j = ch & (nl - 1);
+  const int64_t n0 = (int64_t)blockIdx.x * tpw;
+  const int64_t n = n0 + slot;
+  const bool active = n < N;
+  const double lam = lambdas[j];
+  const double dt = plat.dt, cQ = plat.cQ;
+  const double lt0 = lam * dt;
+  const double Pdt0 = s_Pdt[0], cf0 = Pdt0 + lt0, cf1 = L > 1 ? s_Pdt[1] + lt0 : INFINITY;
+  for (int i = lane; i < kBinChunk * 16; i += 32) (&s_ls[0][0])[i] = 0;  // bytes >= tpw stay 0
+  __syncwarp();
+  // t = 0 runs at r_max (every other level unreachable)
+  double m1, E1, T1;
+  {
+    const double xd = (double)(active ? __ldg(x + n) : 0.0f);
+    const double tau = dt + cQ * q_as_double(xd, s_invB[L - 1]);
+    const double e = s_P[L - 1] * tau;
+    m1 = e + lam * tau;
+    E1 = e;
+    T1 = tau;
+  }
+  bool general = false;
+  const int r_l = lane & (tpw - 1), k_l = lane >> lgtpw, kstride = 32 >> lgtpw;
+  const bool r_ok = n0 + r_l < N;
+  const float* xl = x + (r_ok ? n0 + r_l : 0);
+  const int64_t ldk = (int64_t)kstride * ld;
+  auto stage = [&](int64_t c) {
+    const int64_t t0 = 1 + c * kBinChunk;
+    const float* src = xl + (t0 + k_l) * ld;
+    float* dst = &s_x[c & 1][k_l][r_l];
+    int64_t t = t0 + k_l;
+    for (int i = 0; i < tpw; ++i) {
+      const bool ok = r_ok && t < T;
+      cp_async4z(dst, ok ? src : x, ok);
+      src += ldk;
+      dst += kstride * 16;
+      t += kstride;
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  const int64_t nch = (T - 1 + kBinChunk - 1) / kBinChunk;
+  if (nch > 0) stage(0);
+  for (int64_t c = 0; c < nch; ++c) {
+    if (c + 1 < nch) {
+      stage(c + 1);
+      asm volatile("cp.async.wait_group 1;" ::: "memory");
+    } else {
+      asm volatile("cp.async.wait_group 0;" ::: "memory");
+    }
+    __syncwarp();
+    const int64_t t0 = 1 + c * kBinChunk;
+    const int kn = (int)(T - t0 < kBinChunk ? T - t0 : kBinChunk);
+    // l* of every (step, slot) of the chunk, once
+    const uint32_t a_xc = a_x + (uint32_t)((c & 1) * kBinChunk * 16 * 4);
+    for (int k = k_l; k < kn; k += kstride) {
+      const float xf = lds_f32a(a_xc + (uint32_t)(k * 64 + r_l * 4));
+      int ls = 0;
+      while (ls < L && xf > lds_f32a(a_thr + 4u * ls)) ++ls;  // capacities increase with the level
+      s_ls[k][r_l] = (uint8_t)ls;
+    }
+    __syncwarp();
+    // steps where some trace of the warp is stretched at r_min (bit k)
+    uint32_t slowm;
+    {
+      const uint4 w = *reinterpret_cast<const uint4*>(&s_ls[lane][0]);  // bytes >= tpw stay 0
+      slowm = __ballot_sync(0xFFFFFFFFu, lane < kn && (w.x | w.y | w.z | w.w) != 0u);
+    }
+    // (c, e, tau) of level l at step k of this lane's trace
+    auto level = [&](int k, int l, int ls, double& cl, double& el, double& tl) {
+      if (l < ls) {
+        tl = dt + cQ * q_as_double((double)lds_f32a(a_xc + (uint32_t)(k * 64 + slot * 4)), lds_f64a(a_invB + 8u * l));
+        el = lds_f64a(a_P + 8u * l) * tl;
+        cl = el + lam * tl;
+      } else {
+        tl = dt; el = lds_f64a(a_Pdt + 8u * l);
+        cl = el + lt0;
+      }
+    };
+    bool redo = false;
+    if (!general) {
+      const double m1s = m1, E1s = E1, T1s = T1;
+      bool tie = false;
+      for (int k = 0; k < kn;) {
+        // a run of steps where no trace of the warp is stretched: every
+        // level costs its constant, so the minimum is cf_0 and the runner-up
+        // cf_1 -- three adds and the tie test per step
+        const uint32_t rest = slowm >> k;  // k < 32
+        const int kend = rest ? k + __ffs(rest) - 1 : kn;
+#pragma unroll 4
+        for (; k < kend; ++k) {
+          const double m1n = m1 + cf0;
+          tie |= (m1 + cf1) == m1n;
+          m1 = m1n;
+          E1 = E1 + Pdt0;
+          T1 = T1 + dt;
+        }
+        if (k >= kn) break;
+        const int ls = (int)lds_u8a(a_ls + (uint32_t)(k * 16 + slot));
+        double cmin = INFINITY, c2 = INFINITY, ea = 0.0, ta = 0.0;
+        if (ls < L && h == 0) {  // the lowest unstretched level, and the next one
+          ea = lds_f64a(a_Pdt + 8u * ls);
+          ta = dt;
+          cmin = ea + lt0;
+          if (ls + 1 < L) c2 = lds_f64a(a_Pdt + 8u * (ls + 1)) + lt0;
+        }
+        for (int l = h; l < ls; l += P) {  // stretched levels (rare), this lane's share
+          double cl, el, tl;
+          level(k, l, ls, cl, el, tl);
+          const bool lt = cl < cmin;
+          c2 = lt ? cmin : (cl < c2 ? cl : c2);
+          cmin = lt ? cl : cmin;
+          ea = lt ? el : ea;
+          ta = lt ? tl : ta;
+        }
+#pragma unroll
+        for (int sh = 1; sh < P; sh <<= 1) {  // merge the shares (an exact equality of costs is a tie either way)
+          const double oc = __shfl_xor_sync(0xFFFFFFFFu, cmin, sh), oc2 = __shfl_xor_sync(0xFFFFFFFFu, c2, sh);
+          const double oe = __shfl_xor_sync(0xFFFFFFFFu, ea, sh), ot = __shfl_xor_sync(0xFFFFFFFFu, ta, sh);
+          const bool lt = oc < cmin;
+          const double lose = lt ? cmin : oc;
+          c2 = lose < c2 ? lose : c2;
+          c2 = oc2 < c2 ? oc2 : c2;
+          cmin = lt ? oc : cmin;
+          ea = lt ? oe : ea;
+          ta = lt ? ot : ta;
+        }
+        const double m1n = m1 + cmin;
+        tie |= (m1 + c2) == m1n;  // another level's value equals the minimum
+        m1 = m1n;
+        E1 = E1 + ea;
+        T1 = T1 + ta;
+        ++k;
+      }
+      if (__any_sync(0xFFFFFFFFu, tie)) {
+        m1 = m1s; E1 = E1s; T1 = T1s;
+        redo = true;
+      }
+    }
+    if (general || redo) {
+#pragma unroll 1
+      for (int k = 0; k < kn; ++k) {
+        const int ls = s_ls[k][slot];
+        if (!general) {
+          double cmin = INFINITY, c2 = INFINITY, ea = 0.0, ta = 0.0;
+#pragma unroll
+          for (int l = 0; l < L; ++l) {
+            double cl, el, tl;
+            level(k, l, ls, cl, el, tl);
+            const bool lt = cl < cmin;
+            c2 = lt ? cmin : (cl < c2 ? cl : c2);
+            cmin = lt ? cl : cmin;
+            ea = lt ? el : ea;
+            ta = lt ? tl : ta;
+          }
+          const double m1n = m1 + cmin;
+          if (__any_sync(0xFFFFFFFFu, (m1 + c2) == m1n)) {
+            // a tie: every level's state after this step, the oracle's sums
+#pragma unroll 1
+            for (int l = 0; l < L; ++l) {
+              double cl, el, tl;
+              level(k, l, ls, cl, el, tl);
+              s_V[l][lane] = m1 + cl;
+              s_E[l][lane] = E1 + el;
+              s_T[l][lane] = T1 + tl;
+            }
+            general = true;
+          } else {
+            m1 = m1n;
+            E1 = E1 + ea;
+            T1 = T1 + ta;
+          }
+        } else {
+          // the oracle's recurrence with free switches: best other level o
+          // (lowest on ties), stay when V_l <= V_o
+          int a1 = 0, a2 = 1;
+          if (s_V[1][lane] < s_V[0][lane]) { a1 = 1; a2 = 0; }
+#pragma unroll 1
+          for (int l = 2; l < L; ++l) {
+            const double v = s_V[l][lane];
+            if (v < s_V[a1][lane]) { a2 = a1; a1 = l; }
+            else if (v < s_V[a2][lane]) a2 = l;
+          }
+          const double V1 = s_V[a1][lane], E1o = s_E[a1][lane], T1o = s_T[a1][lane];
+          const double V2 = s_V[a2][lane], E2o = s_E[a2][lane], T2o = s_T[a2][lane];
+#pragma unroll 1
+          for (int l = 0; l < L; ++l) {
+            double cl, el, tl;
+            level(k, l, ls, cl, el, tl);
+            const bool oa = l != a1;  // best other level: a1, or a2 for a1 itself
+            const double vo = oa ? V1 : V2, eo = oa ? E1o : E2o, to = oa ? T1o : T2o;
+            const double v = s_V[l][lane];
+            const bool stay = v <= vo;
+            s_V[l][lane] = (stay ? v : vo) + cl;
+            s_E[l][lane] = (stay ? s_E[l][lane] : eo) + el;
+            s_T[l][lane] = (stay ? s_T[l][lane] : to) + tl;
+          }
+        }
+      }
+    }
+    __syncwarp();  // s_x[c & 1] is restaged by chunk c + 2, s_te / s_ls by the next chunk
+  }
+  if (general) {
+    int b = 0;
+    for (int l = 1; l < L; ++l)
+      if (s_V[l][lane] < s_V[b][lane]) b = l;
+    m1 = s_V[b][lane]; E1 = s_E[b][lane]; T1 = s_T[b][lane];
+  }
+  if (!active || h) return;
+  double* o = out + (n * nl + j) * 3;
+  o[0] = m1;
+  o[1] = E1;
+  o[2] = T1;
+}
+
+#ifndef MAGUS_GRID_P
+#define MAGUS_GRID_P 4  // lanes per (trace, lambda) chain of the free-switch grid DP
+#endif
+constexpr int kGridP = MAGUS_GRID_P;
+
 int launch_bound(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld,
                  const double* lambdas_dev, int32_t nl, bool full_grid, const DevPlatform& plat,
                  double bw_max, double p_lo, double p_span, double* out) {
@@ -861,7 +1148,17 @@ int launch_bound(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t l
   else if (L == 2)  // two levels with switch costs: the branch-free per-step kernel
     bound_binary_kernel<<<blocks, kBoundThreads, 0, s>>>(x, N, T, ld, lambdas_dev, nl, plat, bw_max, p_lo,
                                                          p_span, out);
-  else if (L == 15)
+  else if ((L == 15 || L == 18) && plat.e_sw == 0.0 && plat.t_sw == 0.0 && nl >= 2 && kGridP * nl <= 32 &&
+           32 % (kGridP * nl) == 0) {
+    const int cpw = 32 / kGridP;  // chains per warp
+    const unsigned wb = (unsigned)((N + (cpw / nl) - 1) / (cpw / nl));
+    if (L == 15)
+      bound_grid_free_kernel<15, kGridP><<<wb, 32, 0, s>>>(x, N, T, ld, lambdas_dev, nl, lstep, plat, bw_max, p_lo,
+                                                           p_span, thr, out);
+    else
+      bound_grid_free_kernel<18, kGridP><<<wb, 32, 0, s>>>(x, N, T, ld, lambdas_dev, nl, lstep, plat, bw_max, p_lo,
+                                                           p_span, thr, out);
+  } else if (L == 15)
     bound_dp_kernel<15><<<warps, 32, 0, s>>>(x, N, T, ld, lambdas_dev, nl, lstep, plat, bw_max, p_lo, p_span, thr,
                                              out);
   else if (L == 18)
