@@ -625,7 +625,7 @@ def run_ours(args):
     alone_ms = serial_ms if serial_ms is not None else kern_ms
     alg_bytes = N * T * 4 + (C * N * T / 8 if want_dec else 0)      # per launch on this rank
     traffic = None
-    kname = {1: "ref_kernel", 2: "stream_kernel", 3: "seq_kernel",
+    kname = {1: "ref_kernel", 2: "family_kernel" if st.get("last_family") else "stream_kernel", 3: "seq_kernel",
              4: "walk_map_kernel + walk_replay_kernel + walk_final_kernel",
              5: "spec_kernel + spec_fix_kernel"}.get(st["last_kernel"], "?")
     vtag = {0: "", 1: "_f3", 2: "_f4"}.get(args.variant, f"_v{args.variant}")

@@ -457,6 +457,9 @@ typedef struct {
   int64_t last_reruns;        /* kernel 5: segments whose speculation missed
                                  and were replayed again, in the last replay
                                  (read with a device sync); else 0           */
+  int64_t last_family;        /* stream path: launches of the last replay that
+                                 ran on the family kernel (a sweep grid's
+                                 (W, H) groups; MAGUS_OPT_FAMILY)            */
 } magus_stats;
 /* Per-CTA timeline of the last stream-kernel replay under MAGUS_OPT_TRACE
  * (diagnostics, not the hot path): out host uint64 [cap][8] per CTA (in

@@ -78,7 +78,7 @@ class Stats(ctypes.Structure):
     _fields_ = [("launches_total", ctypes.c_int64), ("main_launches", ctypes.c_int64),
                 ("main_ms_total", ctypes.c_double), ("last_segments", ctypes.c_int64),
                 ("last_kernel", ctypes.c_int64), ("last_grid", ctypes.c_int64),
-                ("last_reruns", ctypes.c_int64)]
+                ("last_reruns", ctypes.c_int64), ("last_family", ctypes.c_int64)]
 
 
 SUMMARY_DT = np.dtype([("n_events", "<i8"), ("n_hi_rounds", "<i8"), ("n_msr_writes", "<i8"),

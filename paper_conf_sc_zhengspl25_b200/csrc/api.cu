@@ -67,7 +67,7 @@ struct magus_ctx_s {
   void* stage_dev = nullptr;
   size_t stage_bytes = 0;
   // stats
-  int64_t launches = 0, main_launches = 0, last_segments = 0, last_kernel = 0, last_grid = 0;
+  int64_t launches = 0, main_launches = 0, last_segments = 0, last_kernel = 0, last_grid = 0, last_family = 0;
   double main_ms = 0.0;
   std::vector<std::pair<cudaEvent_t, cudaEvent_t>> pending;
   std::vector<cudaEvent_t> event_pool;
@@ -909,6 +909,7 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     if (st != MAGUS_OK) return st;
     if (ctx->opt_timing) CK(cudaEventRecord(ev0, ctx->stream));
     int64_t grid_total = 0;
+    ctx->last_family = 0;
     for (size_t gi = 0; gi < ctx->groups.size(); ++gi) {
       auto& g = ctx->groups[gi];
       int grid = 0;
@@ -920,6 +921,7 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
       if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "stream kernel launch");
       launched += r;
       grid_total += grid;
+      if (use_family(ctx, g)) ctx->last_family += 1;
     }
     ctx->last_grid = grid_total;
     if (ctx->opt_timing) CK(cudaEventRecord(ev1, ctx->stream));
@@ -928,6 +930,7 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
   ctx->launches += launched;
   ctx->last_segments = nseg;
   ctx->last_kernel = kernel;
+  if (kernel != 2) ctx->last_family = 0;
   return MAGUS_OK;
 }
 
@@ -1275,6 +1278,7 @@ magus_status magus_get_stats(magus_ctx ctx, magus_stats* out) {
   out->last_kernel = ctx->last_kernel;
   out->last_grid = ctx->last_grid;
   out->last_reruns = 0;
+  out->last_family = ctx->last_family;
   if (ctx->last_kernel == 5 && ctx->spec_reruns) {
     unsigned int r = 0;
     CK(cudaMemcpyAsync(&r, ctx->spec_reruns, sizeof(r), cudaMemcpyDeviceToHost, ctx->stream));

@@ -141,4 +141,12 @@ def test_family_launch_is_used(ctx):
         st = ctx.stats()
         ctx.set_option(magus.OPT_SEGMENTS, 0)
         assert st["launches_total"] - before == nl
+        assert st["last_family"] == nl
         assert st["last_grid"] == grid  # 2 groups of 32 traces x 1 segment per launch
+    ctx.set_option(magus.OPT_FAMILY, 1)
+    try:
+        ctx.replay(xd, magus.grid_fleet64(), want_summary=False, want_base=False)
+        torch.cuda.synchronize()
+        assert ctx.stats()["last_family"] == 0
+    finally:
+        ctx.set_option(magus.OPT_FAMILY, 0)

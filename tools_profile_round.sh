@@ -22,10 +22,10 @@ python bench.py --variant 1 --steps 10 --warmup 3 --no-cpu-baseline --no-e2e > $
 python bench.py --variant 2 --step 2 --steps 10 --warmup 3 --no-cpu-baseline --no-e2e > $O/bench_cfg2_f4.json 2> $O/bench_cfg2_f4.err
 python tools_cta_timeline.py --config 2 --reps 4 > $O/timeline_cfg2.json 2>&1
 ncu --set full --import-source on --clock-control none -k regex:stream_kernel --launch-skip 3 -c 1 -o $O/prof_cfg2 python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-e2e --inflight 1 > $O/ncu_cfg2.log 2>&1
-ncu --set full --import-source on --clock-control none -k regex:stream_kernel --launch-skip 14 -c 1 -o $O/prof_cfg3 python bench.py --config 3 --steps 2 --warmup 3 --no-cpu-baseline --no-e2e --inflight 1 > $O/ncu_cfg3.log 2>&1
+ncu --set full --import-source on --clock-control none -k regex:family_kernel --launch-skip 8 -c 1 -o $O/prof_cfg3 python bench.py --config 3 --steps 2 --warmup 3 --no-cpu-baseline --no-e2e --inflight 1 > $O/ncu_cfg3.log 2>&1
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_cfg2.csv python bench.py --steps 20 --warmup 5 --no-cpu-baseline --no-e2e > /dev/null 2>&1
 ncu --set full --import-source on --clock-control none -k regex:seq_kernel --launch-skip 3 -c 1 -o $O/prof_cfg2_f3 python bench.py --variant 1 --steps 2 --warmup 3 --no-cpu-baseline --no-e2e --inflight 1 > $O/ncu_cfg2_f3.log 2>&1
 ncu --set full --import-source on --clock-control none -k regex:walk_ --launch-skip 9 -c 3 -o $O/prof_cfg2_f4 python bench.py --variant 2 --step 2 --steps 2 --warmup 3 --no-cpu-baseline --no-e2e --inflight 1 > $O/ncu_cfg2_f4.log 2>&1
 ncu --set full --import-source on --clock-control none -k regex:bound_ -c 1 -o $O/prof_cfg2_f2 python bench.py --bound 8 --steps 1 --warmup 3 > $O/ncu_cfg2_f2.log 2>&1
-ncu --set full --import-source on --clock-control none -k regex:bound_dp -c 1 -o $O/prof_cfg2_f2full python bench.py --bound 4 --full-grid --steps 1 --warmup 3 > $O/ncu_cfg2_f2full.log 2>&1
+ncu --set full --import-source on --clock-control none -k regex:bound_grid -c 1 -o $O/prof_cfg2_f2full python bench.py --bound 4 --full-grid --steps 1 --warmup 3 > $O/ncu_cfg2_f2full.log 2>&1
 ls -la $O
