@@ -5,7 +5,8 @@ synccheck / initcheck) runs of the TMA + mbarrier + look-back kernels.
 
 Exercises: several segments (look-back), a ragged trace group and tail word,
 bundles (NB = 4, 128-trace CTAs), one config (the 512-trace CTA), bursts, decisions output, the per-sample kernel, the
-sequential / speculative / walk kernels (level output) and the DP.
+sequential / speculative / walk kernels (level output), the DP kernels and the
+family kernel (a sweep grid's (W, H) group per CTA).
 Exits non-zero if the results disagree with the oracle.
 """
 import os
@@ -79,6 +80,19 @@ def main():
             torch.cuda.synchronize()
             ok &= bool(np.array_equal(out.cpu().numpy()[3, 1],
                                       oracle.offline_bound(x[:200, 3], 100.0, full_grid=full)))
+    # the family kernel (a sweep grid's (W, H) group in one CTA: mask warps,
+    # bundle warps, TMA issued by a mask warp), several segments, decisions
+    fpols = magus.grid_fleet64()
+    fpo = oracle.grid_fleet64()  # the oracle's own restatement of the grid
+    fref = oracle.replay(x, fpo, want_dec=True)
+    with magus.Context(device=0) as ctx:
+        ctx.set_option(magus.OPT_SEGMENTS, 3)
+        r = ctx.replay(xd, fpols, n_traces=N, want_decisions=True)
+        torch.cuda.synchronize()
+        ok &= ctx.stats()["last_family"] == 1
+        ok &= bool(np.array_equal(r.summary_numpy()["energy_j"], fref.summary["energy"]))
+        ok &= bool(np.array_equal(r.summary_numpy()["digest"], fref.summary["digest"]))
+        ok &= bool(np.array_equal(r.decisions_numpy().transpose(0, 2, 1), oracle.decision_words(fref.dec, 8)))
     print("sanitize workload parity:", "ok" if ok else "MISMATCH")
     return 0 if ok else 1
 
