@@ -913,8 +913,11 @@ def run_fleet(args):
             "roofline": {"bound": "alu", "achieved": alu_ach, "peak": alu_peak, "unit": "Gop/s",
                          "frac": alu_ach / alu_peak, "traffic": None,
                          "peak_source": f"148 SMs x 128 lanes x {sm_mhz:.0f} MHz (B200_PROFILING.md unit counts)",
-                         "kernel": "stream_kernel", "kernel_ms": kern_ms / max(1, st["main_launches"]),
-                         "alg_ops_per_decision": 8},
+                         "kernel": "family_kernel" if st.get("last_family") else "stream_kernel",
+                         "kernel_ms": kern_ms / max(1, st["main_launches"]),
+                         "alg_ops_per_decision": 8,
+                         "note": "the 8-op model of SURVEY 8(d) per decision; the kernel shares Alg. 1 work "
+                                 "across the family, so the model rate can exceed the lane peak"},
             "cpu_baseline": cpu,
             "e2e": None, "e2e_note": "the fleet (262 GB) does not fit in host pinned memory; see cfg2 e2e",
             "gpu_launches": int(st["launches_total"]), "clocks": clk,
@@ -955,6 +958,8 @@ def run_bound(args):
     clocks.start()
     time.sleep(0.2)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ctx.reset_stats()
+    ctx.set_option(magus.OPT_TIMING, 1)  # CUDA events around each DP kernel (kernel alone)
     clocks.mark()
     e0.record()
     for _ in range(args.steps):
@@ -964,13 +969,16 @@ def run_bound(args):
     torch.cuda.synchronize()
     clocks.mark()
     clocks.stop()
+    ctx.set_option(magus.OPT_TIMING, 0)
     ms = e0.elapsed_time(e1) / args.steps
+    stb = ctx.stats()
+    kern_ms = stb["main_ms_total"] / max(1, stb["main_launches"])
     units = N * T * len(lams)
     value = units / (ms * 1e-3)
     clk = clocks.summary()
     sm_mhz = clk.get("sm_max_mhz") or 1965.0
     peak = 148 * 64 * sm_mhz * 1e6 / 1e9
-    ach = 12.0 * L * units / (ms * 1e-3) / 1e9
+    ach = 12.0 * L * units / (kern_ms * 1e-3) / 1e9  # the DP's algorithmic fp64 ops / the kernel alone
     # parity of a few traces against the oracle's DP (untimed)
     got = out.cpu().numpy()
     xs = x[:, :4].cpu().numpy()
@@ -983,7 +991,13 @@ def run_bound(args):
                                              "levels": L},
             "roofline": {"bound": "alu", "achieved": ach, "peak": peak, "unit": "Gop/s (fp64)",
                          "frac": ach / peak, "traffic": None, "alg_ops_per_unit_level": 12,
-                         "peak_source": f"148 SMs x 64 fp64 lanes x {sm_mhz:.0f} MHz"},
+                         "peak_source": f"148 SMs x 64 fp64 lanes x {sm_mhz:.0f} MHz",
+                         "kernel_ms": kern_ms, "kernel": {True: "bound_grid_free_kernel / bound_dp_kernel",
+                                                          False: "bound_binary_shared_kernel"}[bool(args.full_grid)],
+                         "method": "the DP's fp64 ops (12 per trace-sample, lambda and level, every level "
+                                   "evaluated) / the kernel's CUDA-event time; the kernels skip most of that "
+                                   "work (one add per step without a tie, DESIGN.md 11), so this is an "
+                                   "algorithmic rate, not the fp64 pipe's utilisation"},
             "gpu_launches": int(ctx.stats()["launches_total"]), "clocks": clk, "parity_sample_ok": bool(parity)}
     print(json.dumps(line), flush=True)
     ctx.close()

@@ -1021,10 +1021,20 @@ magus_status magus_offline_bound(magus_ctx ctx, const float* traces, int64_t N, 
   }
   // pageable source: returns once staged, so `lambdas` may be reused at once
   CK(cudaMemcpyAsync(ctx->lam_dev, lambdas, need, cudaMemcpyHostToDevice, ctx->stream));
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  if (ctx->opt_timing) {  // the DP kernel alone (MAGUS_OPT_TIMING)
+    ev0 = take_event(ctx);
+    ev1 = take_event(ctx);
+    CK(cudaEventRecord(ev0, ctx->stream));
+  }
   const int r = launch_bound(ctx->stream, traces, N, T, ld, (const double*)ctx->lam_dev, nl, full_grid != 0,
                              ctx->dplat, ctx->plat.bw_max_mbs, ctx->plat.p_other_w + ctx->plat.p_unc_min_w,
                              ctx->plat.p_unc_max_w - ctx->plat.p_unc_min_w, out);
   if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "bound kernel launch");
+  if (ctx->opt_timing) {
+    CK(cudaEventRecord(ev1, ctx->stream));
+    ctx->pending.push_back({ev0, ev1});
+  }
   ctx->launches += r;
   return MAGUS_OK;
 }
