@@ -38,6 +38,7 @@
 // the price is reading the traces twice.
 #include <algorithm>
 
+#include "bitops.cuh"
 #include "device_common.cuh"
 
 namespace magus {
@@ -127,6 +128,14 @@ __global__ void __launch_bounds__(kWalkThreads, 5) walk_map_kernel(WalkArgs a, i
   const int K = lmax - lmin;
   const int step = (P.variant & MAGUS_VARIANT_GRADUAL) ? P.step : K;
   HT hist = (HT)history_at(a, P, n, max(t0, P.W)) & hmask;
+  // H <= 32: Alg. 2 bit-parallel per 32-round word (the events of the H
+  // rounds before each position, counted by a carry-save tree / ripple
+  // counter and compared with k), instead of a popcount per round
+  constexpr bool kBits = sizeof(HT) == 4;
+  uint32_t Eprev = kBits ? __brev((uint32_t)hist) : 0u;  // bit i = round t0 - 32 + i
+  uint32_t km[6];
+#pragma unroll
+  for (int j = 0; j < 6; ++j) km[j] = ((P.k >> j) & 1) ? ~0u : 0u;
   int d = 0, lo = lmin, hi = lmax;  // identity (the clamp-shift map l -> min(max(l + d, lo), hi))
   uint32_t* mk = a.mask + (int64_t)cl * 3 * a.nw * a.N + n;
   const int ld32 = (int)a.ld;
@@ -137,11 +146,13 @@ __global__ void __launch_bounds__(kWalkThreads, 5) walk_map_kernel(WalkArgs a, i
   auto round = [&](int i, float xt, float xl) {
     const double D = (double)xt - (double)xl;
     const bool pi = D > P.d_inc, pd = !pi && D < P.d_dec;
-    const bool hf = __popc((uint32_t)(hist & hmask)) + (sizeof(HT) > 4 ? __popc((uint32_t)((uint64_t)hist >> 32)) : 0) >= P.k;
     inc |= (uint32_t)pi << i;
     dcr |= (uint32_t)pd << i;
-    hw |= (uint32_t)hf << i;
-    hist = ((hist << 1) | (HT)(pi || pd)) & hmask;
+    if constexpr (!kBits) {
+      const bool hf = __popc((uint32_t)(hist & hmask)) + __popc((uint32_t)((uint64_t)hist >> 32)) >= P.k;
+      hw |= (uint32_t)hf << i;
+      hist = ((hist << 1) | (HT)(pi || pd)) & hmask;
+    }
   };
   for (int32_t tw = t0; tw < t1; tw += 32) {
     inc = dcr = hw = 0;
@@ -160,6 +171,24 @@ __global__ void __launch_bounds__(kWalkThreads, 5) walk_map_kernel(WalkArgs a, i
     } else {                            // warm-up rounds (t < W) / the ragged tail
       for (int32_t t = max(tw, P.W); t < min(tw + 32, t1); ++t)
         round(t - tw, a.x[(int64_t)t * a.ld + n], a.x[(int64_t)(t - P.W + 1) * a.ld + n]);
+    }
+    if constexpr (kBits) {
+      // rounds of this word that ran Alg. 2: t >= W and t < t1 (inc / dcr
+      // are zero elsewhere, so E = inc | dcr is the event log of the word)
+      const uint32_t E = inc | dcr;
+      uint32_t valid = ~0u;
+      if (tw < P.W) valid = (P.W - tw >= 32) ? 0u : (~0u << (P.W - tw));
+      if (tw + 32 > t1) valid &= (1u << (t1 - tw)) - 1u;
+      if (P.H == 10) {
+        uint32_t cnt[4];
+        Window<10>::count(E, Eprev, 10, cnt);
+        hw = ge_k<4>(cnt, km) & valid;
+      } else {
+        uint32_t cnt[6];
+        Window<0>::count(E, Eprev, P.H, cnt);
+        hw = ge_k<6>(cnt, km) & valid;
+      }
+      Eprev = E;
     }
     const int64_t w = tw >> 5;
     mk[w * a.N] = inc;
