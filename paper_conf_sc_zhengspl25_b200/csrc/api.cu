@@ -910,6 +910,10 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     if (ctx->opt_timing) CK(cudaEventRecord(ev0, ctx->stream));
     int64_t grid_total = 0;
     ctx->last_family = 0;
+    for (auto& g : ctx->groups)  // one launch per group: its CTAs index grid.x
+      if (group_ctas(ctx, N, g, nseg) > (int64_t)INT32_MAX)
+        return fail(ctx, MAGUS_ERR_UNSUPPORTED, "%lld CTAs in one launch exceed the grid limit; replay fewer traces",
+                    (long long)group_ctas(ctx, N, g, nseg));
     for (size_t gi = 0; gi < ctx->groups.size(); ++gi) {
       auto& g = ctx->groups[gi];
       int grid = 0;
