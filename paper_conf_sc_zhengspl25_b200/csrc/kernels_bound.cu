@@ -781,8 +781,7 @@ bound_binary_shared_kernel(const float* __restrict__ x, int64_t N, int64_t T, in
           T1 = T1 + (up ? b.x : a.x);
         }
       } else {
-#pragma unroll 8
-        for (int k = 0; k < kn; ++k) {
+        auto step0 = [&](int k) {
           const double2 a = s_te[k][slot][0];
           const double c0 = a.y + lam * a.x;
           const bool up = cf1 < c0;
@@ -790,6 +789,13 @@ bound_binary_shared_kernel(const float* __restrict__ x, int64_t N, int64_t T, in
           m1 = m1 + (up ? cf1 : c0);
           E1 = E1 + (up ? Pdt1 : a.y);
           T1 = T1 + (up ? dt : a.x);
+        };
+        if (kn == kBinChunk) {  // every chunk but the last: straight-line code
+#pragma unroll
+          for (int k = 0; k < kBinChunk; ++k) step0(k);
+        } else {
+#pragma unroll 8
+          for (int k = 0; k < kn; ++k) step0(k);
         }
       }
       if (__any_sync(0xFFFFFFFFu, tie)) {
