@@ -891,7 +891,9 @@ bound_grid_free_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_
   __shared__ float s_x[2][kBinChunk][16];       // [buffer][step][trace slot]
   __shared__ __align__(16) uint8_t s_ls[kBinChunk][16];  // l* of (step, slot)
   __shared__ double s_invB[L], s_P[L], s_Pdt[L];
-  __shared__ double s_V[L][32], s_E[L][32], s_T[L][32];  // per-level state after a tie (rare)
+  // per-level state after a tie (rare): per-thread local memory, so the
+  // CTA's shared memory stays small enough for every warp to be resident
+  double s_Vl[L], s_El[L], s_Tl[L];
   __shared__ float s_thr[32];
   const int lane = threadIdx.x;
   for (int i = lane; i < L; i += 32) {
@@ -1074,9 +1076,9 @@ bound_grid_free_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_
             for (int l = 0; l < L; ++l) {
               double cl, el, tl;
               level(k, l, ls, cl, el, tl);
-              s_V[l][lane] = m1 + cl;
-              s_E[l][lane] = E1 + el;
-              s_T[l][lane] = T1 + tl;
+              s_Vl[l] = m1 + cl;
+              s_El[l] = E1 + el;
+              s_Tl[l] = T1 + tl;
             }
             general = true;
           } else {
@@ -1088,26 +1090,26 @@ bound_grid_free_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_
           // the oracle's recurrence with free switches: best other level o
           // (lowest on ties), stay when V_l <= V_o
           int a1 = 0, a2 = 1;
-          if (s_V[1][lane] < s_V[0][lane]) { a1 = 1; a2 = 0; }
+          if (s_Vl[1] < s_Vl[0]) { a1 = 1; a2 = 0; }
 #pragma unroll 1
           for (int l = 2; l < L; ++l) {
-            const double v = s_V[l][lane];
-            if (v < s_V[a1][lane]) { a2 = a1; a1 = l; }
-            else if (v < s_V[a2][lane]) a2 = l;
+            const double v = s_Vl[l];
+            if (v < s_Vl[a1]) { a2 = a1; a1 = l; }
+            else if (v < s_Vl[a2]) a2 = l;
           }
-          const double V1 = s_V[a1][lane], E1o = s_E[a1][lane], T1o = s_T[a1][lane];
-          const double V2 = s_V[a2][lane], E2o = s_E[a2][lane], T2o = s_T[a2][lane];
+          const double V1 = s_Vl[a1], E1o = s_El[a1], T1o = s_Tl[a1];
+          const double V2 = s_Vl[a2], E2o = s_El[a2], T2o = s_Tl[a2];
 #pragma unroll 1
           for (int l = 0; l < L; ++l) {
             double cl, el, tl;
             level(k, l, ls, cl, el, tl);
             const bool oa = l != a1;  // best other level: a1, or a2 for a1 itself
             const double vo = oa ? V1 : V2, eo = oa ? E1o : E2o, to = oa ? T1o : T2o;
-            const double v = s_V[l][lane];
+            const double v = s_Vl[l];
             const bool stay = v <= vo;
-            s_V[l][lane] = (stay ? v : vo) + cl;
-            s_E[l][lane] = (stay ? s_E[l][lane] : eo) + el;
-            s_T[l][lane] = (stay ? s_T[l][lane] : to) + tl;
+            s_Vl[l] = (stay ? v : vo) + cl;
+            s_El[l] = (stay ? s_El[l] : eo) + el;
+            s_Tl[l] = (stay ? s_Tl[l] : to) + tl;
           }
         }
       }
@@ -1117,8 +1119,8 @@ bound_grid_free_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_
   if (general) {
     int b = 0;
     for (int l = 1; l < L; ++l)
-      if (s_V[l][lane] < s_V[b][lane]) b = l;
-    m1 = s_V[b][lane]; E1 = s_E[b][lane]; T1 = s_T[b][lane];
+      if (s_Vl[l] < s_Vl[b]) b = l;
+    m1 = s_Vl[b]; E1 = s_El[b]; T1 = s_Tl[b];
   }
   if (!active || h) return;
   double* o = out + (n * nl + j) * 3;
@@ -1128,7 +1130,7 @@ bound_grid_free_kernel(const float* __restrict__ x, int64_t N, int64_t T, int64_
 }
 
 #ifndef MAGUS_GRID_P
-#define MAGUS_GRID_P 4  // lanes per (trace, lambda) chain of the free-switch grid DP
+#define MAGUS_GRID_P 8  // most lanes per (trace, lambda) chain of the free-switch grid DP
 #endif
 constexpr int kGridP = MAGUS_GRID_P;
 
@@ -1154,16 +1156,25 @@ int launch_bound(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t l
   else if (L == 2)  // two levels with switch costs: the branch-free per-step kernel
     bound_binary_kernel<<<blocks, kBoundThreads, 0, s>>>(x, N, T, ld, lambdas_dev, nl, plat, bw_max, p_lo,
                                                          p_span, out);
-  else if ((L == 15 || L == 18) && plat.e_sw == 0.0 && plat.t_sw == 0.0 && nl >= 2 && kGridP * nl <= 32 &&
-           32 % (kGridP * nl) == 0) {
-    const int cpw = 32 / kGridP;  // chains per warp
-    const unsigned wb = (unsigned)((N + (cpw / nl) - 1) / (cpw / nl));
-    if (L == 15)
-      bound_grid_free_kernel<15, kGridP><<<wb, 32, 0, s>>>(x, N, T, ld, lambdas_dev, nl, lstep, plat, bw_max, p_lo,
-                                                           p_span, thr, out);
-    else
-      bound_grid_free_kernel<18, kGridP><<<wb, 32, 0, s>>>(x, N, T, ld, lambdas_dev, nl, lstep, plat, bw_max, p_lo,
-                                                           p_span, thr, out);
+  else if ((L == 15 || L == 18) && plat.e_sw == 0.0 && plat.t_sw == 0.0 && nl >= 2 && nl <= 16 &&
+           32 % nl == 0) {
+    // lanes per chain: as many as the warp allows up to kGridP (more lanes
+    // split a slow step's stretched levels further; measured best at 8 for
+    // the mix traces, 18.3 vs 21.4 ms at 4)
+    const int P = std::min(kGridP, 32 / nl);
+    const unsigned wb = (unsigned)((N + (32 / P / nl) - 1) / (32 / P / nl));
+    auto go = [&](auto kern) {
+      kern<<<wb, 32, 0, s>>>(x, N, T, ld, lambdas_dev, nl, lstep, plat, bw_max, p_lo, p_span, thr, out);
+    };
+    if (L == 15) {
+      if (P >= 8) go(bound_grid_free_kernel<15, 8>);
+      else if (P == 4) go(bound_grid_free_kernel<15, 4>);
+      else go(bound_grid_free_kernel<15, 2>);
+    } else {
+      if (P >= 8) go(bound_grid_free_kernel<18, 8>);
+      else if (P == 4) go(bound_grid_free_kernel<18, 4>);
+      else go(bound_grid_free_kernel<18, 2>);
+    }
   } else if (L == 15)
     bound_dp_kernel<15><<<warps, 32, 0, s>>>(x, N, T, ld, lambdas_dev, nl, lstep, plat, bw_max, p_lo, p_span, thr,
                                              out);

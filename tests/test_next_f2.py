@@ -123,7 +123,7 @@ def test_gpu_offline_bound_bit_exact(full_grid, r_max):
 @pytest.mark.gpu
 @pytest.mark.parametrize("full_grid", [False, True])
 @pytest.mark.parametrize("case", ["free_switch", "flat_power_ties", "tiny_switch", "adversarial", "short"])
-@pytest.mark.parametrize("nl", [3, 8])
+@pytest.mark.parametrize("nl", [3, 4, 8])
 def test_gpu_offline_bound_modes_bit_exact(full_grid, case, nl):
     """The throughput kernel's two bookkeeping modes: free
     switches (the paper's default: scalar path sums), equal power at every
@@ -140,9 +140,11 @@ def test_gpu_offline_bound_modes_bit_exact(full_grid, case, nl):
     plat.p_unc_min_w = kw.get("p_unc_min", plat.p_unc_min_w)
     plat.p_unc_max_w = kw.get("p_unc_max", plat.p_unc_max_w)
     plat_o = oracle.platform(**kw)
-    # 8 lambdas: a warp holds whole traces (the binary kernel's shared
-    # per-(trace, step) model-M terms); 3: traces straddle warps
-    lams = [0.0, 25.0, 400.0] if nl == 3 else [0.0, 10.0, 25.0, 40.0, 160.0, 400.0, 2560.0, 1e6]
+    # 4 / 8 lambdas: a warp holds whole traces (the binary kernel's shared
+    # per-(trace, step) model-M terms; the free-switch grid kernel with 8 /
+    # 4 lanes per chain); 3: traces straddle warps (the generic kernels)
+    lams = {3: [0.0, 25.0, 400.0], 4: [0.0, 25.0, 400.0, 1e6],
+            8: [0.0, 10.0, 25.0, 40.0, 160.0, 400.0, 2560.0, 1e6]}[nl]
     Ts = [1, 2, 33, 34] if case == "short" else [1999]
     kind = gen.KIND_ADVERSARIAL if case == "adversarial" else gen.KIND_MIX
     with magus.Context(device=0, platform=plat) as ctx:
