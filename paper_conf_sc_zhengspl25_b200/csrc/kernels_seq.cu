@@ -40,7 +40,8 @@
 #include "device_common.cuh"
 
 #ifndef SEQ_ABLATE
-#define SEQ_ABLATE 0  // developer timing experiments: 1 no accounting, 2 no producer math, 3 no chain
+#define SEQ_ABLATE 0  // developer timing experiments, a bit mask: 1 no accounting, 2 no producer math,
+                      // 4 no chain, 8 no producer loads (constant samples)
 #endif
 
 namespace magus {
@@ -230,6 +231,14 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
       const uint32_t mdfs = word_mdfs(jj, live) >> (16 * h), lv = live >> (16 * h);
       const float* src = xcol + t0 * a.ld;
       const float* lsrc = xcol + (t0 - W + 1) * a.ld;
+      if (SEQ_ABLATE & 8) {
+#pragma unroll
+        for (int u = 0; u < 16; ++u) {
+          xv[u] = (float)(lane + u);
+          lg[u] = (float)(lane + 2 * u);
+        }
+        return;
+      }
       if (__all_sync(0xFFFFFFFFu, (mdfs & 0xFFFFu) == 0xFFFFu)) {
 #pragma unroll
         for (int u = 0; u < 16; ++u) {
@@ -271,7 +280,7 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
         const uint32_t rd16 = (mdfs >> (16 * h)) & 0xFFFFu;
         uint32_t b16 = 0, bm16 = 0, r16 = 0, i16 = 0, d16 = 0, cw = 0;
 #pragma unroll
-        for (int u = 0; u < 16; ++u) {
+        for (int u = 0; u < ((SEQ_ABLATE & 2) ? 0 : 16); ++u) {
           const float xt = cx[u];
           b16 |= (uint32_t)(xt > xthr) << u;
           bm16 |= (uint32_t)(xt > xthrM) << u;
@@ -338,7 +347,7 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
       const uint32_t live = cnt == 32 ? 0xFFFFFFFFu : ((1u << cnt) - 1u);
       const uint32_t mdfs = word_mdfs(j, live);
       const bool fast = narrow && __all_sync(0xFFFFFFFFu, mdfs == 0xFFFFFFFFu);
-      if (SEQ_ABLATE == 3) { warp_arrive(done(s)); continue; }
+      if (SEQ_ABLATE & 4) { warp_arrive(done(s)); continue; }
       const uint32_t* pm = reinterpret_cast<const uint32_t*>(sl + kOffPM) + lane;
       const uint32_t inc = pm[2 * kLanes], dcr = pm[3 * kLanes];
       uint32_t decm = 0, m1 = 0, evm = 0, him = 0;   // m1: binary leff mask / MULTI change mask
@@ -530,7 +539,7 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
   for (int64_t j = acc_id; j < nwords; j += kAccountants) {
     const int s = (int)(j % kSlots);
     mb_wait(done(s), (uint32_t)((j / kSlots) & 1));
-    if (SEQ_ABLATE == 1) { release(j); continue; }
+    if (SEQ_ABLATE & 1) { release(j); continue; }
     const unsigned char* sl = slots + s * kSlotBytes;
     const int64_t t0 = j * kWord;
     const int cnt = word_cnt(j);
