@@ -462,7 +462,7 @@ def run_ours(args):
     if args.burst > 0:  # NEXT f1: Sec. 6.3 burst Jaccard counters in the same pass
         plat.burst_mbs = args.burst
     opts = [(magus.OPT_WAVES, args.waves), (magus.OPT_SEGMENTS, args.segments), (magus.OPT_BUNDLE, args.bundle),
-            (magus.OPT_SPEC_WARM, args.spec_warm), (magus.OPT_KERNEL, args.kernel)]
+            (magus.OPT_SPEC_WARM, args.spec_warm), (magus.OPT_KERNEL, args.kernel), (magus.OPT_WALK1, args.walk1)]
     ctx = magus.Context(device=local, stream=stream, platform=plat)
     for k, v in opts:
         if v:
@@ -629,7 +629,8 @@ def run_ours(args):
     alg_bytes = N * T * 4 + (C * N * T / 8 if want_dec else 0)      # per launch on this rank
     traffic = None
     kname = {1: "ref_kernel", 2: "family_kernel" if st.get("last_family") else "stream_kernel", 3: "seq_kernel",
-             4: "walk_map_kernel + walk_replay_kernel + walk_final_kernel",
+             4: ("walk_fused_kernel + walk_final_kernel" if args.walk1
+                 else "walk_map_kernel + walk_replay_kernel + walk_final_kernel"),
              5: "spec_kernel + spec_fix_kernel"}.get(st["last_kernel"], "?")
     vtag = {0: "", 1: "_f3", 2: "_f4"}.get(args.variant, f"_v{args.variant}")
     # traffic only from an ncu capture of this very kernel and workload
@@ -1026,6 +1027,7 @@ def main():
     ap.add_argument("--step", type=int, default=1, help="ratio step of the gradual variant")
     ap.add_argument("--spec-warm", type=int, default=0, help="f3 speculation warm-up rounds (0 auto)")
     ap.add_argument("--kernel", type=int, default=0, help="MAGUS_OPT_KERNEL (0 auto; 5 = speculative f3)")
+    ap.add_argument("--walk1", type=int, default=0, help="MAGUS_OPT_WALK1: 1 = the one-pass f4 walk (A/B)")
     ap.add_argument("--cpu-threads", type=int, default=0, help="host threads of the oracle legs (0 = all cores)")
     ap.add_argument("--comm", choices=["torch", "native"], default="torch",
                     help="the totals all-reduce: torch.distributed NCCL, or the library's own (magus_comm_init)")

@@ -437,6 +437,13 @@ enum {
                                  128-trace CTAs (4 per SM) instead of the
                                  default 512-trace CTA per SM (A/B option;
                                  results are identical)                      */
+  MAGUS_OPT_WALK1 = 9,        /* 1: the open-loop walk (kernel 4) in ONE pass
+                                 (segment map and replay in the same scan,
+                                 the carry-dependent prefix replayed after a
+                                 decoupled look-back) instead of the default
+                                 two passes (maps, then the replay); measured
+                                 slower on config 2; A/B
+                                 option, results identical                  */
   MAGUS_OPT_FAMILY = 8        /* 0 (default): a (W, H) group of <= 16 bundles
                                  of 4 configs with <= 8 distinct tau_inc and
                                  tau_dec thresholds (a sweep grid, Sec. 6.4)

@@ -26,6 +26,7 @@ PLATFORM_INTEL_A100, PLATFORM_INTEL_MAX1550 = 0, 1
 GEN_MIX, GEN_ADVERSARIAL = 0, 1
 OPT_KERNEL, OPT_SEGMENTS, OPT_TIMING, OPT_WAVES, OPT_BUNDLE, OPT_SPEC_WARM, OPT_TRACE, OPT_NARROW = 0, 1, 2, 3, 4, 5, 6, 7
 OPT_FAMILY = 8
+OPT_WALK1 = 9
 KERNEL_AUTO, KERNEL_REFERENCE, KERNEL_STREAM, KERNEL_SEQUENTIAL, KERNEL_WALK, KERNEL_SPEC = 0, 1, 2, 3, 4, 5
 TOT_WORDS = 18
 TOT_NAMES = ["n_traces", "n_viol", "events", "hi_rounds", "msr_writes", "changes", "min_dec",

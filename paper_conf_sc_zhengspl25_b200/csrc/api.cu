@@ -26,6 +26,7 @@ struct magus_ctx_s {
   int sms = 148;
   // options
   int64_t opt_kernel = 0, opt_segments = 0, opt_timing = 0, opt_waves = 0, opt_trace = 0, opt_narrow = 0;
+  int64_t opt_walk1 = 0;   // 1: the one-pass walk kernel (A/B)
   int64_t opt_family = 0;  // 0: family kernel for the groups it takes; 1: bundle kernels only
   void* trace_dev = nullptr;   // MAGUS_OPT_TRACE timeline [trace_cap][8]
   int64_t trace_cap = 0, trace_n = 0;
@@ -568,6 +569,9 @@ magus_status magus_set_option(magus_ctx ctx, int32_t key, int64_t value) {
     case MAGUS_OPT_NARROW:
       ctx->opt_narrow = value ? 1 : 0;
       return MAGUS_OK;
+    case MAGUS_OPT_WALK1:
+      ctx->opt_walk1 = value ? 1 : 0;
+      return MAGUS_OK;
     case MAGUS_OPT_FAMILY:
       ctx->opt_family = value ? 1 : 0;
       return MAGUS_OK;
@@ -770,7 +774,7 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     const double p_lo = ctx->plat.p_other_w + ctx->plat.p_unc_min_w;
     const double p_span = ctx->plat.p_unc_max_w - ctx->plat.p_unc_min_w;
     int r = launch_walk(ctx->stream, traces, N, T, ld, dev_policies(ctx), C, max_H, ctx->dplat, ctx->plat.bw_max_mbs,
-                        p_lo, p_span, nseg, seg_len, sp, summ, base, out_decisions, out_levels);
+                        p_lo, p_span, nseg, seg_len, sp, summ, base, out_decisions, out_levels, ctx->opt_walk1 != 0);
     if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "walk kernel launch");
     launched += r;
     ctx->last_grid = ((N + 127) / 128) * nseg * C;

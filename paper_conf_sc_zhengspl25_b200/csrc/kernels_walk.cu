@@ -390,6 +390,291 @@ __global__ void __launch_bounds__(kWalkThreads) walk_final_kernel(WalkArgs a, De
   so->energy_j = energy + plat.e_sw * (double)changes;
 }
 
+
+// ---------------------------------------------------------------------------
+// One pass (walk_fused_kernel): the map and the replay of a segment in the
+// same scan, carry by decoupled look-back.
+//
+// Every round applies a clamp-shift map with the offset dl in {+K (the
+// override, l.10: min(l + K, r_max) = r_max), +step, -step, 0}, so one
+// thread walks three values per round: the level reached from r_max (hi),
+// from r_min (lo) and the saturated offset d.  The clamp-shift maps are
+// monotone, so every carry-in gives a level between lo and hi: once lo == hi
+// (after an override, or after the steps saturate at a bound) the level is
+// the same for every carry-in and equals hi.  From the word after that point
+// on, the thread meters model M on the fly; the words before it (the
+// carry-dependent prefix, usually short) keep their Alg. 1 / Alg. 2 masks in
+// scratch and are replayed from the true carry once the look-back has it.
+// The segment's status is its map (lo == hi: the end level itself).
+// Work tickets are taken in (config, segment, trace group) order, so every
+// predecessor segment holds a CTA already: the look-back never waits on a
+// CTA that is not running.
+// ---------------------------------------------------------------------------
+constexpr uint32_t kWalkPub = 1u << 24;  // status published (map in bits 0..23)
+
+struct FusedArgs {
+  uint32_t* status;   // [C][nseg][N] (zero at launch)
+  uint32_t* ticket;   // [batches] (zero at launch)
+  int32_t ngroups;    // trace groups of kWalkThreads
+};
+
+__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_u32(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+template <typename HT, bool BURST>
+__global__ void __launch_bounds__(kWalkThreads, 4) walk_fused_kernel(WalkArgs a, DevPlatform plat,
+                                                                  const __grid_constant__ WalkLevels lv,
+                                                                  FusedArgs f, int32_t batch) {
+  __shared__ double s_invB[kWalkMaxLv];
+  __shared__ float s_xthr[kWalkMaxLv];
+  __shared__ uint8_t s_bkeep[kWalkMaxLv];
+  __shared__ uint8_t s_lv[32][kWalkThreads];  // dec[32w + i] of the current word
+  __shared__ uint32_t s_ticket;
+  extern __shared__ unsigned int s_cnt[];     // [nlev][kWalkThreads] intervals per level
+  const int lmin = plat.r_min, lmax = plat.r_max, nlev = lmax - lmin + 1;
+  const int tid = threadIdx.x;
+  for (int i = 0; i < nlev; ++i) s_cnt[i * kWalkThreads + tid] = 0u;
+  for (int i = tid; i < nlev; i += kWalkThreads) {
+    s_invB[i] = lv.invB[i];
+    s_xthr[i] = lv.xthr[i];
+    s_bkeep[i] = lv.bkeep[i];
+  }
+  if (tid == 0) s_ticket = atomicAdd(f.ticket + batch, 1u);
+  __syncthreads();
+  const uint32_t per_cfg = (uint32_t)a.nseg * (uint32_t)f.ngroups;
+  const int32_t cl = (int32_t)(s_ticket / per_cfg);
+  const int32_t s = (int32_t)((s_ticket % per_cfg) / (uint32_t)f.ngroups);
+  const int32_t g = (int32_t)(s_ticket % (uint32_t)f.ngroups);
+  const int32_t c = a.c0 + cl;
+  const int64_t n = (int64_t)g * kWalkThreads + tid;
+  if (n >= a.N) return;
+  const DevPolicy P = a.pol[c];
+  const int32_t t0 = s * a.seg_len, t1 = min(a.T, t0 + a.seg_len);
+  const int K = lmax - lmin;
+  const int step = (P.variant & MAGUS_VARIANT_GRADUAL) ? P.step : K;
+  const HT hmask = P.H >= (int)(8 * sizeof(HT)) ? (HT)~(HT)0 : (HT)(((HT)1 << P.H) - 1);
+  HT hist = (HT)history_at(a, P, n, max(t0, P.W)) & hmask;
+  constexpr bool kBits = sizeof(HT) == 4;
+  uint32_t Eprev = kBits ? __brev((uint32_t)hist) : 0u;  // bit i = round t0 - 32 + i
+  uint32_t km[6];
+#pragma unroll
+  for (int j = 0; j < 6; ++j) km[j] = ((P.k >> j) & 1) ? ~0u : 0u;
+  const int ld32 = (int)a.ld;
+  const float xthr_max = plat.xthr_max, xburst = plat.xburst;
+  const double invB_max = plat.invB_max;
+  unsigned int* lvn = a.lvn + (int64_t)c * nlev * a.N + n;
+  unsigned long long* lvq = a.lvq + (int64_t)c * nlev * a.N + n;
+  uint32_t* mk = a.mask + (int64_t)cl * 3 * a.nw * a.N + n;
+
+  // the three walks (segment 0 starts from the known dec[-1] = r_max)
+  int lh = lmax, ll = s == 0 ? lmax : lmin, dd = 0;
+  int32_t t_live = s == 0 ? t0 : -1;   // first interval metered in the scan (-1: none yet)
+  // model-M state of the metered intervals
+  int cur = lmax;                      // level of the current run of intervals
+  int32_t run_start = t0;
+  int qlev = lmax;                     // stretch q of level qlev not yet flushed
+  unsigned long long qacc = 0, q_base = 0, digest = 0;
+  int32_t events = 0, hi_rounds = 0, msr = 0, changes = 0, n_min_dec = 0, b_base = 0, b_magus = 0;
+
+  // The replay of one word at the level `lvl` (dec[32w - 1]) with model M:
+  // the step rule from the masks, the per-interval flags, and the sparse
+  // stretch / run-length / burst work over the word's set bits.
+  auto meter_word = [&](int32_t tw, uint32_t inc, uint32_t dcr, uint32_t hw, const float (&xs)[32], int& lvl) {
+    const int64_t w = tw >> 5;
+    const int rem = min(32, t1 - tw);
+    const uint32_t live = rem == 32 ? ~0u : ((1u << rem) - 1u);
+    const int before = lvl;
+    uint32_t word = 0, chg = 0, big = 0, bmx = 0, bst = 0;
+    float xthr_cur = s_xthr[lvl - lmin];
+#pragma unroll
+    for (int i = 0; i < 32; ++i) {
+      big |= (uint32_t)(xs[i] > xthr_cur) << i;   // stretched at its level dec[t-1]
+      bmx |= (uint32_t)(xs[i] > xthr_max) << i;
+      if (BURST) bst |= (uint32_t)(xs[i] > xburst) << i;
+      const int dl = ((hw >> i) & 1u) ? K : (((inc >> i) & 1u) ? step : (((dcr >> i) & 1u) ? -step : 0));
+      const int prev = lvl;
+      lvl = min(max(lvl + dl, lmin), lmax);        // l.10 / l.18-19 / l.23-25
+      s_lv[i][tid] = (uint8_t)lvl;
+      xthr_cur = s_xthr[lvl - lmin];
+      word |= (uint32_t)(lvl == lmin) << i;
+      chg |= (uint32_t)(lvl != prev) << i;
+    }
+    word &= live;
+    big &= live;
+    bmx &= live;
+    bst &= live;
+    n_min_dec += __popc(word);
+    changes += __popc(chg);                       // rounds past T hold: no change
+    if (a.dec) a.dec[((int64_t)c * a.nw + w) * a.N + n] = word;
+    digest += (unsigned long long)word * digest_mul(w);
+    if (a.levels)
+      for (int i = 0; i < rem; ++i) a.levels[((int64_t)c * a.T + tw + i) * a.N + n] = s_lv[i][tid];
+    uint32_t m = big | bmx | bst;
+    while (m) {
+      const int i = __ffs(m) - 1;
+      m &= m - 1;
+      const int L = i ? (int)s_lv[i - 1][tid] : before;
+      const float xt = __ldg(a.x + (int64_t)(tw + i) * a.ld + n);
+      if ((big >> i) & 1u) {
+        if (L != qlev) {
+          if (qacc) atomicAdd(lvq + (int64_t)(qlev - lmin) * a.N, qacc);
+          qacc = 0;
+          qlev = L;
+        }
+        qacc += q_literal(xt, s_invB[L - lmin]);
+      }
+      if ((bmx >> i) & 1u) q_base += q_literal(xt, invB_max);
+      if (BURST && ((bst >> i) & 1u)) {
+        ++b_base;
+        b_magus += s_bkeep[L - lmin];
+      }
+    }
+    m = chg;
+    while (m) {
+      const int i = __ffs(m) - 1;
+      m &= m - 1;
+      s_cnt[(cur - lmin) * kWalkThreads + tid] += (unsigned int)(tw + i + 1 - run_start);
+      run_start = tw + i + 1;
+      cur = s_lv[i][tid];
+    }
+  };
+
+  for (int32_t tw = t0; tw < t1; tw += 32) {
+    // ---- Alg. 1 (and Alg. 2 for H > 32) over the word ----
+    float xs[32];
+    uint32_t inc = 0, dcr = 0, hw = 0;
+    const float* px = a.x + (int64_t)tw * a.ld + n;
+    auto round = [&](int i, float xt, float xl) {
+      const double D = (double)xt - (double)xl;
+      const bool pi = D > P.d_inc, pd = !pi && D < P.d_dec;
+      inc |= (uint32_t)pi << i;
+      dcr |= (uint32_t)pd << i;
+      if constexpr (!kBits) {
+        const bool hf = __popc((uint32_t)(hist & hmask)) + __popc((uint32_t)((uint64_t)hist >> 32)) >= P.k;
+        hw |= (uint32_t)hf << i;
+        hist = ((hist << 1) | (HT)(pi || pd)) & hmask;
+      }
+    };
+    if (tw >= P.W && tw + 32 <= t1) {   // a full word of MDFS rounds
+      const float* pl = px - (int64_t)(P.W - 1) * a.ld;
+#pragma unroll
+      for (int h = 0; h < 4; ++h) {
+        float xl[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) xs[h * 8 + i] = __ldg(px + (h * 8 + i) * ld32);
+        load_rows<8>(pl + h * 8 * ld32, ld32, xl);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) round(h * 8 + i, xs[h * 8 + i], xl[i]);
+      }
+    } else {                            // warm-up rounds (t < W) / the ragged tail
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        const int32_t t = tw + i;
+        xs[i] = t < t1 ? __ldg(px + i * ld32) : 0.0f;
+        if (t >= P.W && t < t1) round(i, xs[i], __ldg(a.x + (int64_t)(t - P.W + 1) * a.ld + n));
+      }
+    }
+    if constexpr (kBits) {   // Alg. 2 bit-parallel (E = the word's event log)
+      const uint32_t E = inc | dcr;
+      uint32_t valid = ~0u;
+      if (tw < P.W) valid = (P.W - tw >= 32) ? 0u : (~0u << (P.W - tw));
+      if (tw + 32 > t1) valid &= (1u << (t1 - tw)) - 1u;
+      if (P.H == 10) {
+        uint32_t cnt[4];
+        Window<10>::count(E, Eprev, 10, cnt);
+        hw = ge_k<4>(cnt, km) & valid;
+      } else {
+        uint32_t cnt[6];
+        Window<0>::count(E, Eprev, P.H, cnt);
+        hw = ge_k<6>(cnt, km) & valid;
+      }
+      Eprev = E;
+    }
+    events += __popc(inc | dcr);                   // l.17 / l.22
+    hi_rounds += __popc(hw);
+    msr += __popc(inc | dcr | hw);                 // tune_uncore_freq calls
+    // ---- the step rule ----
+    if (t_live >= 0) {
+      meter_word(tw, inc, dcr, hw, xs, lh);        // levels known: replay and meter
+    } else {
+      // carry-dependent: walk the three values, keep the masks for the replay
+      const int64_t w = tw >> 5;
+      mk[w * a.N] = inc;
+      mk[(a.nw + w) * a.N] = dcr;
+      mk[(2 * (int64_t)a.nw + w) * a.N] = hw;
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        const int dl = ((hw >> i) & 1u) ? K : (((inc >> i) & 1u) ? step : (((dcr >> i) & 1u) ? -step : 0));
+        lh = min(max(lh + dl, lmin), lmax);
+        ll = min(max(ll + dl, lmin), lmax);
+        dd = min(max(dd + dl, -K), K);
+      }
+      if (ll == lh && tw + 32 < t1) {              // collapsed: meter from the next word on
+        t_live = tw + 32;
+        cur = qlev = lh;
+        run_start = t_live;
+      }
+    }
+  }
+  // ---- publish the segment's map, look back for the carry ----
+  uint32_t* st = f.status + ((int64_t)cl * a.nseg) * a.N + n;
+  const bool known = t_live >= 0 || ll == lh;
+  st_release_u32(st + (int64_t)s * a.N, kWalkPub | (known ? map_pack(0, lh, lh) : map_pack(dd, ll, lh)));
+  if (t_live >= 0) s_cnt[(cur - lmin) * kWalkThreads + tid] += (unsigned int)(t1 - run_start);
+  const int32_t t_def = t_live >= 0 ? t_live : t1;   // intervals [t0, t_def) replayed from the carry
+  if (s > 0 && t_def > t0) {
+    int32_t j = s - 1;
+    uint32_t v;
+    for (;; --j) {   // the nearest predecessor whose end level is known (segment 0's always is)
+      while (((v = ld_acquire_u32(st + (int64_t)j * a.N)) & kWalkPub) == 0u) __nanosleep(64);
+      if (((v >> 8) & 0xFFu) == ((v >> 16) & 0xFFu)) break;
+    }
+    int lvl = (int)((v >> 16) & 0xFFu);
+    for (++j; j < s; ++j) lvl = map_apply(ld_acquire_u32(st + (int64_t)j * a.N), lvl);
+    if (!known)   // the true end level, for the segments after this one
+      st_release_u32(st + (int64_t)s * a.N, kWalkPub | map_pack(0, map_apply(map_pack(dd, ll, lh), lvl),
+                                                                  map_apply(map_pack(dd, ll, lh), lvl)));
+    // replay the carry-dependent words from the true carry
+    if (qacc) atomicAdd(lvq + (int64_t)(qlev - lmin) * a.N, qacc);
+    qacc = 0;
+    cur = qlev = lvl;
+    run_start = t0;
+    for (int32_t tw = t0; tw < t_def; tw += 32) {
+      const int64_t w = tw >> 5;
+      const uint32_t inc = mk[w * a.N], dcr = mk[(a.nw + w) * a.N], hw = mk[(2 * (int64_t)a.nw + w) * a.N];
+      const float* px = a.x + (int64_t)tw * a.ld + n;
+      float xs[32];
+#pragma unroll
+      for (int i = 0; i < 32; ++i) xs[i] = tw + i < t1 ? __ldg(px + i * ld32) : 0.0f;
+      meter_word(tw, inc, dcr, hw, xs, lvl);
+    }
+    s_cnt[(cur - lmin) * kWalkThreads + tid] += (unsigned int)(t_def - run_start);
+  }
+  for (int l = 0; l < nlev; ++l) {
+    const unsigned int v = s_cnt[l * kWalkThreads + tid];
+    if (v) atomicAdd(lvn + (int64_t)l * a.N, v);
+  }
+  if (qacc) atomicAdd(lvq + (int64_t)(qlev - lmin) * a.N, qacc);
+  unsigned long long* acc = a.acc + (int64_t)c * kWalkFields * a.N + n;
+#ifdef WALK_STATS  // developer statistics in the burst fields: deferred words, look-back steps
+  b_base = (t_def - t0 + 31) / 32;
+  b_magus = s > 0 && t_def > t0 ? 1 : 0;
+#endif
+  const unsigned long long vals[kWalkFields] = {
+      (unsigned long long)events, (unsigned long long)hi_rounds, (unsigned long long)msr,
+      (unsigned long long)changes, (unsigned long long)n_min_dec, q_base, digest,
+      (unsigned long long)b_base, (unsigned long long)b_magus};
+#pragma unroll
+  for (int fi = 0; fi < kWalkFields; ++fi)
+    if (vals[fi]) atomicAdd(acc + (int64_t)fi * a.N, vals[fi]);
+}
+
 }  // namespace
 
 // configs per launch: the pass-1 masks of a batch stay below this
@@ -405,13 +690,13 @@ size_t walk_scratch_bytes(int64_t N, int32_t C, int64_t T, int64_t nseg, const D
   const int64_t B = walk_batch(N, C, T), nw = (T + 31) / 32;
   auto al = [](size_t b) { return (b + 255) / 256 * 256; };
   return al(4 * (size_t)B * nseg * N) + al(12 * (size_t)B * nw * N) + al(8 * (size_t)C * kWalkFields * N) +
-         al(4 * (size_t)C * nlev * N) + al(8 * (size_t)C * nlev * N);
+         al(4 * (size_t)C * nlev * N) + al(8 * (size_t)C * nlev * N) + al(4 * (size_t)((C + B - 1) / B));
 }
 
 int launch_walk(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld, const DevPolicy* pol_dev,
                 int32_t C, int32_t max_H, const DevPlatform& plat, double bw_max, double p_lo, double p_span,
                 int64_t nseg, int64_t seg_len, void* scratch, magus_summary* out_summary, magus_base* out_base,
-                uint32_t* out_dec, uint8_t* out_levels) {
+                uint32_t* out_dec, uint8_t* out_levels, bool fused) {
   const int nlev = plat.r_max - plat.r_min + 1;
   const int64_t B = walk_batch(N, C, T), nw = (T + 31) / 32;
   auto al = [](size_t b) { return (b + 255) / 256 * 256; };
@@ -436,6 +721,8 @@ int launch_walk(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld
   a.lvn = (unsigned int*)sp;
   sp += al(4 * (size_t)C * nlev * N);
   a.lvq = (unsigned long long*)sp;
+  sp += al(8 * (size_t)C * nlev * N);
+  uint32_t* tickets = (uint32_t*)sp;
   a.summary = out_summary;
   a.base = out_base;
   a.dec = out_dec;
@@ -461,7 +748,30 @@ int launch_walk(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld
             cudaSuccess)
       return -1;
   }
-  for (int64_t c0 = 0; c0 < C; c0 += B) {
+  if (fused) {
+    // one pass: the accumulators and the batch tickets start at zero, the
+    // status words of every batch too (cleared before each batch)
+    const int64_t nb = (C + B - 1) / B;
+    if (cudaMemsetAsync(a.acc, 0, (size_t)((char*)tickets - (char*)a.acc) + 4 * (size_t)nb, s) != cudaSuccess) return -1;
+    auto fk = max_H > 32 ? (plat.burst_on ? walk_fused_kernel<uint64_t, true> : walk_fused_kernel<uint64_t, false>)
+                         : (plat.burst_on ? walk_fused_kernel<uint32_t, true> : walk_fused_kernel<uint32_t, false>);
+    if (cnt_smem > 48 * 1024 &&
+        cudaFuncSetAttribute(fk, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cnt_smem) != cudaSuccess)
+      return -1;
+    FusedArgs fa;
+    fa.status = a.map;
+    fa.ticket = tickets;
+    fa.ngroups = (int32_t)((N + kWalkThreads - 1) / kWalkThreads);
+    for (int64_t c0 = 0, bi = 0; c0 < C; c0 += B, ++bi) {
+      a.c0 = (int32_t)c0;
+      const int64_t nc = std::min<int64_t>(B, C - c0);
+      if (cudaMemsetAsync(a.map, 0, 4 * (size_t)nc * nseg * N, s) != cudaSuccess) return -1;
+      const unsigned grid = (unsigned)(fa.ngroups * nseg * nc);
+      fk<<<grid, kWalkThreads, cnt_smem, s>>>(a, plat, lv, fa, (int32_t)bi);
+      launched += 1;
+    }
+  }
+  for (int64_t c0 = 0; c0 < C && !fused; c0 += B) {
     a.c0 = (int32_t)c0;
     const dim3 grid((unsigned)((N + kWalkThreads - 1) / kWalkThreads), (unsigned)nseg,
                     (unsigned)std::min<int64_t>(B, C - c0));

@@ -27,10 +27,11 @@ magus = pytest.importorskip("paper_conf_sc_zhengspl25_b200")
 from test_gpu_seq import FIELDS, _check, _opol, _platforms  # noqa: E402
 
 
-def _levels(ctx, x, pols, segments=0, kernel=4):
+def _levels(ctx, x, pols, segments=0, kernel=4, walk1=0):
     xd = torch.from_numpy(np.ascontiguousarray(x)).cuda()
     ctx.set_option(magus.OPT_KERNEL, kernel)
     ctx.set_option(magus.OPT_SEGMENTS, segments)
+    ctx.set_option(magus.OPT_WALK1, walk1)
     try:
         lv, res = ctx.replay_levels(xd, pols)
         torch.cuda.synchronize()
@@ -38,6 +39,7 @@ def _levels(ctx, x, pols, segments=0, kernel=4):
     finally:
         ctx.set_option(magus.OPT_KERNEL, magus.KERNEL_AUTO)
         ctx.set_option(magus.OPT_SEGMENTS, 0)
+        ctx.set_option(magus.OPT_WALK1, 0)
     return lv.cpu().numpy().transpose(0, 2, 1), res      # [C, N, T]
 
 
@@ -46,9 +48,10 @@ MIXED = [  # (variant, step) of each config in ONE launch
 ]
 
 
+@pytest.mark.parametrize("walk1", [0, 1])
 @pytest.mark.parametrize("mix", range(len(MIXED)))
 @pytest.mark.parametrize("segments", [0, 1, 3, 11, 87])
-def test_walk_kernel_vs_oracle(mix, segments):
+def test_walk_kernel_vs_oracle(mix, segments, walk1):
     N, T = 190, 2777            # 87 segments of 32 steps: every word its own segment
     x = gen.gen_traces(gen.SEEDS[1], N, T)
     pols = []
@@ -58,18 +61,36 @@ def test_walk_kernel_vs_oracle(mix, segments):
     po, pm = _platforms("a100", 12000.0)
     ref = oracle.replay(x, _opol(pols), po, want_dec=True)
     with magus.Context(device=0, platform=pm) as ctx:
-        lv, res = _levels(ctx, x, pols, segments)
+        lv, res = _levels(ctx, x, pols, segments, walk1=walk1)
     _check(lv, res, ref, po, T, len(pols))
 
 
+@pytest.mark.parametrize("walk1", [0, 1])
+@pytest.mark.parametrize("segments", [0, 11, 87])
+def test_walk_kernel_carry_dependent_segments(segments, walk1):
+    """No override (t_hi = 2: s/H >= 2 never holds) and +-1 steps over a
+    14-ratio range: a segment's map rarely becomes constant, so the one-pass
+    kernel replays long carry-dependent prefixes (often whole segments) after
+    the look-back, through chains of non-constant predecessor maps."""
+    N, T = 160, 2777
+    x = gen.gen_traces(gen.SEEDS[3], N, T)
+    pols = [magus.make_policy(variant=2, step=1, t_hi=2.0), magus.make_policy(W=4, H=7, t_hi=2.0, variant=2, step=2)]
+    po, pm = _platforms("a100", 12000.0)
+    ref = oracle.replay(x, _opol(pols), po, want_dec=True)
+    with magus.Context(device=0, platform=pm) as ctx:
+        lv, res = _levels(ctx, x, pols, segments, walk1=walk1)
+    _check(lv, res, ref, po, T, len(pols))
+
+
+@pytest.mark.parametrize("walk1", [0, 1])
 @pytest.mark.parametrize("N,T,segments", [(33, 17, 0), (1, 1, 0), (1, 10000, 0), (1, 10000, 300), (129, 64, 2)])
-def test_walk_kernel_shapes(N, T, segments):
+def test_walk_kernel_shapes(N, T, segments, walk1):
     x = gen.gen_traces(gen.SEEDS[2], N, T)
     pols = [magus.make_policy(variant=2, step=1), magus.make_policy(variant=0)]
     po, pm = _platforms("a100", 12000.0)
     ref = oracle.replay(x, _opol(pols), po, want_dec=True)
     with magus.Context(device=0, platform=pm) as ctx:
-        lv, res = _levels(ctx, x, pols, segments)
+        lv, res = _levels(ctx, x, pols, segments, walk1=walk1)
     _check(lv, res, ref, po, T, len(pols))
 
 
