@@ -37,6 +37,7 @@
 // exact for every double; model M uses the literal quantiser q_literal of
 // device_common.cuh.  ref_kernel (kernels_ref.cu) keeps the printed
 // divisions and is the parity baseline this kernel is tested against.
+#include "bitops.cuh"
 #include "device_common.cuh"
 
 #ifndef SEQ_ABLATE
@@ -61,8 +62,8 @@ constexpr int kMaxLv = 128;
 
 // slot layout (bytes)
 constexpr int kOffX = 0;                              // float [32 steps][32 lanes] samples
-constexpr int kOffCode = kOffX + 4 * kWord * kLanes;  // u32 [8][32] closed-binary outcome codes
-constexpr int kOffPM = kOffCode + 4 * 8 * kLanes;     // u32 [5][32] big, burst, inc, dec, big-at-max
+constexpr int kOffCode = kOffX + 4 * kWord * kLanes;  // u32 [16][32] closed-binary transition codes (2 steps per word)
+constexpr int kOffPM = kOffCode + 4 * 16 * kLanes;    // u32 [5][32] big, burst, inc, dec, big-at-max
 constexpr int kOffCM = kOffPM + 4 * 5 * kLanes;       // u32 [5][32] dec, leff|change, event, hi masks, dec[t0-1]
 constexpr int kOffLv = kOffCM + 4 * 5 * kLanes;       // u8 [32][32] MULTI ratios dec[t0+i]
 constexpr int kOffL = kOffLv + kWord * kLanes;        // float [32][32] Alg. 1 lags (CLOSED && MULTI)
@@ -97,6 +98,43 @@ __device__ __forceinline__ void mb_wait(uint32_t bar, uint32_t parity) {
 __device__ __forceinline__ void warp_arrive(uint32_t bar) {
   __syncwarp();
   mb_arrive(bar);
+}
+
+// The closed binary loop's transition code of one round (16 bits), from the
+// four Alg. 1 differences d[a*2+b] (a = interval t at r_min, b = the lag
+// interval t-W+1 at r_min).  Byte b (the lag's level) holds, for the level
+// lm of interval t (= dec[t-1]): bit 4*lm = the next decision is min (lm = 0:
+// -1 and not +1, Alg. 3 l.25; lm = 1: not +1, l.18 -- both unless hi, l.10),
+// bit 4*lm + 1 = an event (+1 or -1 logged, l.17/22).  The consumer picks
+// the byte by the lag's level and the nibble by lm with one LOP3.
+__device__ __forceinline__ void code_bits(uint32_t& c, double d, double d_inc, double d_dec, uint32_t dnb,
+                                          uint32_t ev, uint32_t stay) {
+  // -1 (d < d_dec): set dnb (stay | ev for lm = 0, ev for lm = 1, whose stay
+  // bit is preset); then +1 (d > d_inc): set ev, clear stay.  NaN: neither.
+  asm("{\n.reg .pred p, q;\nsetp.lt.f64 p, %1, %2;\nsetp.gt.f64 q, %1, %3;\n@p or.b32 %0, %0, %4;\n"
+      "@q lop3.b32 %0, %0, %5, %6, 0x54;\n}"
+      : "+r"(c) : "d"(d), "d"(d_dec), "d"(d_inc), "r"(dnb), "r"(ev), "r"(stay));
+}
+// the 16-bit code of one round from the samples of intervals t and t-W+1
+// (delivered = min(x, capacity) at each of the two levels, model M)
+__device__ __forceinline__ uint32_t closed_code(float xt, float xl, double Bmin, double Bmax, bool capfree,
+                                                double d_inc, double d_dec) {
+  const double vt = (double)xt, vl = (double)xl;
+  const double ytm = vt > Bmin ? Bmin : vt, ylm = vl > Bmin ? Bmin : vl;
+  const double ytM = capfree ? vt : (vt > Bmax ? Bmax : vt), ylM = capfree ? vl : (vl > Bmax ? Bmax : vl);
+  uint32_t c = 0x1010u;                                    // lm = 1: stays min unless +1
+  code_bits(c, ytM - ylM, d_inc, d_dec, 0x0003u, 0x0002u, 0x0001u);   // a = 0, b = 0
+  code_bits(c, ytM - ylm, d_inc, d_dec, 0x0300u, 0x0200u, 0x0100u);   // a = 0, b = 1
+  code_bits(c, ytm - ylM, d_inc, d_dec, 0x0020u, 0x0020u, 0x0010u);   // a = 1, b = 0
+  code_bits(c, ytm - ylm, d_inc, d_dec, 0x2000u, 0x2000u, 0x1000u);   // a = 1, b = 1
+  return c;
+}
+
+template <uint32_t LUT>
+__device__ __forceinline__ uint32_t lop3(uint32_t a, uint32_t b, uint32_t c) {
+  uint32_t d;
+  asm("lop3.b32 %0, %1, %2, %3, %4;" : "=r"(d) : "r"(a), "r"(b), "r"(c), "n"(LUT));
+  return d;
 }
 
 // delivered throughput of model M at capacity B (oracle `observed`)
@@ -220,6 +258,7 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
       }
     };
     const float xthrM = plat.xthr_max;  // x <= xthrM: no stretch at r_max
+    const float xobsM = closed ? plat.xobs_max : INFINITY;   // x > xobsM <=> (double)x > B_max
     // Half-word pipeline: the 32 loads of the next half (this word's second
     // half, or the first half of this producer's next word) are in flight
     // while the current half is evaluated.
@@ -279,22 +318,33 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
         }
         const uint32_t rd16 = (mdfs >> (16 * h)) & 0xFFFFu;
         uint32_t b16 = 0, bm16 = 0, r16 = 0, i16 = 0, d16 = 0, cw = 0;
+        // no sample of the half above the capacity at r_max (the common case):
+        // delivered = x there, two fewer selects per sample
+        bool capfree = false;
+        if constexpr (CLOSED && !MULTI) {
+          float mx = cx[0];
+#pragma unroll
+          for (int u = 0; u < 16; ++u) mx = fmaxf(mx, fmaxf(cx[u], cl[u]));
+          capfree = __all_sync(0xFFFFFFFFu, !(mx > xobsM));   // NaN: delivered = NaN either way
+        }
 #pragma unroll
         for (int u = 0; u < ((SEQ_ABLATE & 2) ? 0 : 16); ++u) {
           const float xt = cx[u];
-          b16 |= (uint32_t)(xt > xthr) << u;
-          bm16 |= (uint32_t)(xt > xthrM) << u;
-          r16 |= (uint32_t)(xt > xburst) << u;
-          if (!(CLOSED && MULTI) && ((rd16 >> u) & 1)) {
+          or_if_gt(b16, xt, xthr, 1u << u);
+          or_if_gt(bm16, xt, xthrM, 1u << u);
+          or_if_gt(r16, xt, xburst, 1u << u);
+          if constexpr (CLOSED && !MULTI) {
+            // every round (the consumer reads the codes of MDFS rounds only)
+            cw |= closed_code(xt, cl[u], obs_min, obs_max, capfree, d_inc, d_dec) << (16 * (u & 1));
+            if (u & 1) {
+              cwp[(8 * h + (u >> 1)) * kLanes] = cw;
+              cw = 0;
+            }
+          } else if (!(CLOSED && MULTI) && ((rd16 >> u) & 1)) {
             uint32_t cd = 0, up = 0, dn = 0;
             eval(xt, cl[u], cd, up, dn);
-            cw |= cd << (8 * (u & 3));
             i16 |= up << u;
             d16 |= dn << u;
-          }
-          if (CLOSED && !MULTI && (u & 3) == 3) {
-            cwp[(4 * h + (u >> 2)) * kLanes] = cw;
-            cw = 0;
           }
         }
         big |= b16 << (16 * h);
@@ -331,7 +381,7 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
     const int wsh = (int)(W - 1) & 63;
     // branch-free 32-bit words when every lane has W, H <= 32 and the word is
     // all MDFS rounds (everything but a trace's first and last word)
-    const bool narrow = __all_sync(0xFFFFFFFFu, !active || (W <= 32 && P.H <= 32));
+    const bool narrow = __all_sync(0xFFFFFFFFu, !active || (W <= 32 && P.H <= 32 && (!CLOSED || (W >= 3 && P.H >= 2))));
     const uint32_t hmask32 = (uint32_t)hmask;
     uint64_t hist = 0;               // uncore_tune_ls: H zeros (P@24182); bit j = round t-1-j
     int s_cnt = 0;                   // popc(hist)
@@ -359,21 +409,66 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
           // steps bit i is step i
           const uint32_t* cwp = reinterpret_cast<const uint32_t*>(sl + kOffCode) + lane;
           uint32_t h = (uint32_t)hist, lb = (uint32_t)lvb, iv = inc, dv = dcr;
+          if constexpr (CLOSED) {
+            // The chain of a round is two LOP3: the code nibble picked by the
+            // level of interval t (LM, all ones at r_min) and the override
+            // (lt = !hi, Alg. 2 as the sign of D = s - k).  Everything else
+            // accumulates by multiply-adds (the FMA pipe, next to the ALU
+            // pipe's LOP3 / shifts), in reversed bit order (bit 31 = round 0).
+            // lag interval of the NEXT round = bit W-3 of lb before this
+            // round's push (W >= 3), the outgoing event of the next round =
+            // bit H-2 of h before the push (H >= 2): both read from registers
+            // this round's decision does not write (off the chain)
+            const uint32_t wsh2 = (uint32_t)(W - 3), hsh2 = (uint32_t)(hsh - 1);
+            uint32_t lag = (lb >> (wsh2 + 1)) & 1u, out = (h >> hsh) & 1u;
+            uint32_t LM = 0u - lm;
+            int D = s_cnt - k;                          // hi <=> s >= k <=> D >= 0
+            uint32_t lt = (uint32_t)D >> 31;
+            uint32_t dacc = 0, eacc = 0, lacc = 0;
+            const uint32_t lm0 = lm;
+            uint32_t wa = cwp[0], wb = cwp[kLanes];
+#pragma unroll 1
+            for (int g = 0; g < kWord / 4; ++g) {
+              const uint32_t w0 = wa, w1 = wb;
+              if (g < kWord / 4 - 1) {
+                wa = cwp[(2 * g + 2) * kLanes];
+                wb = cwp[(2 * g + 3) * kLanes];
+              }
+#pragma unroll
+              for (int u = 0; u < 4; ++u) {
+                const uint32_t w = u < 2 ? w0 : w1;
+                const uint32_t P = w >> (16 * (u & 1) + 8 * lag);     // byte of the lag's level
+                const uint32_t V = lop3<0xD8>(P, P >> 4, LM);           // nibble of interval t's level
+                const uint32_t nlm = lop3<0x80>(V, lt, 1u);             // l.10 override, else l.18 / l.25 / hold
+                const uint32_t e = (V >> 1) & 1u;                       // l.17 / l.22 event
+                D += (int)e - (int)out;
+                lag = (lb >> wsh2) & 1u;
+                out = (h >> hsh2) & 1u;
+                lacc = lacc * 2u + lt;
+                lt = (uint32_t)D >> 31;
+                lb = lb * 2u + (LM & 1u);
+                h = h * 2u + e;
+                eacc = eacc * 2u + e;
+                LM = 0u - nlm;
+                dacc = dacc * 2u + nlm;
+              }
+            }
+            decm = __brev(dacc);
+            evm = __brev(eacc);
+            him = ~__brev(lacc);
+            m1 = (decm << 1) | lm0;                     // interval t runs at dec[t-1] (reading R6)
+            lm = LM & 1u;
+            s_cnt = D + k;
+            hist = h & hmask32;
+            lvb = lb;
+          } else {
 #pragma unroll 1
           for (int g = 0; g < kWord / 4; ++g) {
-            const uint32_t cw = CLOSED ? cwp[g * kLanes] : 0u;
 #pragma unroll
             for (int u = 0; u < 4; ++u) {
               m1 = __funnelshift_r(m1, lm, 1);      // interval t runs at dec[t-1] (reading R6)
               uint32_t up, dn, e;
-              if constexpr (CLOSED) {
-                lb = (lb << 1) | lm;
-                const uint32_t idx = 2u * lm + ((lb >> wsh) & 1u);
-                const uint32_t cd = (cw >> (8 * u)) >> idx;
-                up = cd & 1u;
-                dn = (cd >> 4) & 1u;
-                e = (cd & 0x11u) != 0u;
-              } else {
+              {
                 up = iv & 1u;
                 dn = dv & 1u;
                 iv >>= 1;
@@ -392,7 +487,7 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
             }
           }
           hist = h;
-          lvb = lb;
+          }
         } else {
 #pragma unroll 1
           for (int i = 0; i < kWord; ++i) {
@@ -401,20 +496,19 @@ __global__ void __launch_bounds__(kThreads) seq_kernel(SeqArgs a, DevPlatform pl
               if constexpr (CLOSED) lvb = (lvb << 1) | lm;
               if ((mdfs >> i) & 1) {
                 uint32_t e, up, dn;
-                if constexpr (CLOSED) {
-                  const uint32_t idx = 2u * lm + (uint32_t)((lvb >> wsh) & 1ULL);
-                  const uint32_t cw = reinterpret_cast<const uint32_t*>(sl + kOffCode)[(i >> 2) * kLanes + lane];
-                  const uint32_t cd = (cw >> (8 * (i & 3))) >> idx;
-                  up = cd & 1u;
-                  dn = (cd >> 4) & 1u;
-                  e = (cd & 0x11u) != 0u;
+                const uint32_t hi = s_cnt >= k;
+                if constexpr (CLOSED) {   // closed_code: byte by the lag's level, nibble by lm
+                  const uint32_t lag = (uint32_t)((lvb >> wsh) & 1ULL);
+                  const uint32_t cw = reinterpret_cast<const uint32_t*>(sl + kOffCode)[(i >> 1) * kLanes + lane];
+                  const uint32_t V = (cw >> (16 * (i & 1) + 8 * lag)) >> (4 * lm);
+                  e = (V >> 1) & 1u;
+                  lm = hi ? 0u : (V & 1u);
                 } else {
                   up = (inc >> i) & 1u;
                   dn = (dcr >> i) & 1u;
                   e = up | dn;
+                  lm = (hi | up) ? 0u : (dn | lm);
                 }
-                const uint32_t hi = s_cnt >= k;
-                lm = (hi | up) ? 0u : (dn | lm);
                 him |= hi << i;
                 const int out = (int)((hist >> hsh) & 1ULL);
                 hist = ((hist << 1) | e) & hmask;

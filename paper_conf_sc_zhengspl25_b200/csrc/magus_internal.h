@@ -45,7 +45,7 @@ struct DevPlatform {
   float xburst;                  // x > xburst <=> (double)x > theta
   int32_t burst_on;              // theta > 0 and B_max > theta
   int32_t burst_min_keeps;       // B_min > theta: the level never hides a burst
-  int32_t pad_;
+  float xobs_max;                // x > xobs_max <=> (double)x > B_max (f3: delivered < x at r_max)
 };
 
 // Work/scratch block of the fused stream kernel (kernels_stream.cu).  The

@@ -187,6 +187,7 @@ DevPlatform make_dev_platform(const magus_platform& p) {
   d.Bmin = Bmin;
   d.Bmax = Bmax;
   d.xburst = above_threshold(p.burst_mbs);
+  d.xobs_max = above_threshold(Bmax);
   d.burst_on = (p.burst_mbs > 0.0 && Bmax > p.burst_mbs) ? 1 : 0;
   d.burst_min_keeps = (Bmin > p.burst_mbs) ? 1 : 0;
   return d;
