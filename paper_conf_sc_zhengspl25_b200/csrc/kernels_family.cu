@@ -88,7 +88,14 @@ __device__ __forceinline__ unsigned long long lds_u64v(uint32_t a) {
 
 // sum of q over the positions of `lv` (any mask), from the word's inclusive
 // prefix P (column `col`, row stride 256 B): sum_t lv_t (P_t - P_t-1) = sum
-// over run ends P_end - sum over the positions just before a run start
+// over run ends P_end - sum over the positions just before a run start.
+// q is zero where the sample does not stretch (P flat there), so only lv's
+// bits at the stretched positions matter: the callers pass lv held forward
+// from one stretched position to the next (the carry-chain sample-and-hold of
+// bitops.cuh), whose runs change only where lv changes between consecutive
+// stretched samples -- never more runs than lv, one run (one load) for a
+// word whose stretched samples are all in lv; the loop's trip count is the
+// maximum over the warp's lanes.
 __device__ __forceinline__ unsigned long long run_sum(uint32_t lv, uint32_t col) {
   const uint32_t nx = lv >> 1;
   uint32_t plus = lv & ~nx, minus = ~lv & nx;
@@ -454,13 +461,13 @@ family_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
 #pragma unroll
       for (int k = 0; k < kFNB; ++k) {
         const uint32_t lq = Lvk[k] & outm;
-        if (lq & smin) qmin[k] += run_sum(lq, pcol);
+        if (lq & smin) qmin[k] += run_sum(forward_fill(smin, lq, 0u), pcol);
       }
       if (xmx) {  // some sample exceeds even the capacity at max (rare)
 #pragma unroll
         for (int k = 0; k < kFNB; ++k) {
           const uint32_t lx = ~Lvk[k] & outm;
-          if (lx & xmx) FS(k, tidb).qmax += run_sum(lx, pxcol);
+          if (lx & xmx) FS(k, tidb).qmax += run_sum(forward_fill(xmx, lx, 0u), pxcol);
         }
       }
       Gb += Pw;
