@@ -58,15 +58,17 @@ def main():
         vpo = oracle.policies([dict(W=p.window, H=p.history, L=p.deriv_len, tau_inc=p.tau_inc, tau_dec=p.tau_dec,
                                     t_hi=p.t_hi, variant=p.variant, step=p.step) for p in vpols])
         vref = oracle.replay(x, vpo, oracle.platform(burst=12000.0), want_dec=True)
-        runs = [(magus.KERNEL_SEQUENTIAL, vpols[:1], [0], 0),        # f3: seq_kernel<closed, binary>
-                (magus.KERNEL_SEQUENTIAL, vpols, [0, 1, 2], 0),      # mixed: seq_kernel<closed, multi>
-                (magus.KERNEL_SPEC, vpols[:1], [0], 7),
-                (magus.KERNEL_WALK, vpols[1:], [1, 2], 6)]
+        runs = [(magus.KERNEL_SEQUENTIAL, vpols[:1], [0], 0, 0),        # f3: seq_kernel<closed, binary>
+                (magus.KERNEL_SEQUENTIAL, vpols, [0, 1, 2], 0, 0),      # mixed: seq_kernel<closed, multi>
+                (magus.KERNEL_SPEC, vpols[:1], [0], 7, 0),
+                (magus.KERNEL_WALK, vpols[1:], [1, 2], 6, 0),
+                (magus.KERNEL_WALK, vpols[1:], [1, 2], 6, 1)]           # the one-pass walk (OPT_WALK1)
         only = os.environ.get("SANITIZE_ONLY")  # e.g. "0,2,3": a subset of the runs above
         if only:
             runs = [runs[int(i)] for i in only.split(",")]
-        for kernel, pp, idx, segs in runs:
+        for kernel, pp, idx, segs, walk1 in runs:
             ctx.set_option(magus.OPT_KERNEL, kernel)
+            ctx.set_option(magus.OPT_WALK1, walk1)
             ctx.set_option(magus.OPT_SEGMENTS, segs)
             ctx.set_option(magus.OPT_SPEC_WARM, 1)
             lv, rr = ctx.replay_levels(xd, pp, n_traces=N)
@@ -75,6 +77,7 @@ def main():
             ok &= bool(np.array_equal(rr.summary_numpy()["energy_j"], vref.summary["energy"][idx]))
         ctx.set_option(magus.OPT_KERNEL, magus.KERNEL_AUTO)
         ctx.set_option(magus.OPT_SEGMENTS, 0)
+        ctx.set_option(magus.OPT_WALK1, 0)
         for full in (False, True):  # f2: the scalar-path binary kernel, the two-lane grid kernel
             out = ctx.offline_bound(xd[:200, :8], [0.0, 100.0], full_grid=full)
             torch.cuda.synchronize()

@@ -20,6 +20,7 @@ python bench.py --bound 8 --steps 5 --warmup 3 > $O/bench_cfg2_f2.json 2> $O/ben
 python bench.py --bound 4 --full-grid --steps 3 --warmup 3 > $O/bench_cfg2_f2full.json 2> $O/bench_cfg2_f2full.err
 python bench.py --variant 1 --steps 10 --warmup 3 --no-cpu-baseline --no-e2e > $O/bench_cfg2_f3.json 2> $O/bench_cfg2_f3.err
 python bench.py --variant 2 --step 2 --steps 10 --warmup 3 --no-cpu-baseline --no-e2e > $O/bench_cfg2_f4.json 2> $O/bench_cfg2_f4.err
+python bench.py --variant 2 --step 2 --steps 10 --warmup 3 --no-cpu-baseline --no-e2e --walk1 1 > $O/bench_cfg2_f4_walk1.json 2> $O/bench_cfg2_f4_walk1.err
 python tools_cta_timeline.py --config 2 --reps 4 > $O/timeline_cfg2.json 2>&1
 ncu --set full --import-source on --clock-control none -k regex:stream_kernel --launch-skip 3 -c 1 -o $O/prof_cfg2 python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-e2e --inflight 1 > $O/ncu_cfg2.log 2>&1
 ncu --set full --import-source on --clock-control none -k regex:family_kernel --launch-skip 8 -c 1 -o $O/prof_cfg3 python bench.py --config 3 --steps 2 --warmup 3 --no-cpu-baseline --no-e2e --inflight 1 > $O/ncu_cfg3.log 2>&1
