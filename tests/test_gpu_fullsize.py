@@ -6,7 +6,9 @@ their exact integer words on the sampled subset by partition invariance).
   config 3  4,096 x 100,000 x SWEEP256 (4 W-group launches, bundles of 4)
   config 4  one GPU's shard at 8 GPUs: 8,192 x 1,000,000 x FLEET64, one shot
   config 5  16,384 adversarial x 1,000,000 x paper_default
-  config 2  f4 gradual through the walk kernels (143 segments)
+  config 2  f4 gradual through the walk kernels (143 segments), and through
+            the one-pass walk kernel (MAGUS_OPT_WALK1)
+  config 2  f3 closed loop through the sequential kernel (transition codes)
 
 Config 2 (paper's rule) is in test_gpu_parity.py; config 4 through the
 time-chunked path is sampled by bench.py (parity_sample_ok) and by
@@ -114,3 +116,43 @@ def test_full_config2_gradual_sweep_in_config_batches(ctx):
     torch.cuda.synchronize()
     assert ctx.stats()["last_kernel"] == magus.KERNEL_WALK
     _check_sample(ctx, xd, pols, np.array([0, 1, 2047, N - 1]), r)
+
+
+def test_full_config2_gradual_one_pass_walk_sampled(ctx):
+    """The one-pass walk kernel (decoupled look-back, carry-dependent prefixes
+    replayed) at the bench's size and segmentation."""
+    N, T = 4096, 100_000
+    xd = ctx.gen_traces(gen.SEEDS[2], N, T)
+    pols = [magus.make_policy(variant=2, step=2)]
+    ctx.set_option(magus.OPT_WALK1, 1)
+    try:
+        r = ctx.replay(xd, pols, want_decisions=True)
+        torch.cuda.synchronize()
+    finally:
+        ctx.set_option(magus.OPT_WALK1, 0)
+    assert ctx.stats()["last_kernel"] == magus.KERNEL_WALK
+    sample = _sample(N, 12, 5)
+    _check_sample(ctx, xd, pols, sample, r)
+    xs = xd[:, torch.as_tensor(sample, device=xd.device)].cpu().numpy()
+    ref = oracle.replay(np.ascontiguousarray(xs), to_oracle_policies(pols), want_dec=True)
+    dec = r.decisions_numpy()
+    for i, n in enumerate(sample):
+        assert np.array_equal(dec[0, :, n], oracle.decision_words(ref.dec[0, i], 8)), n
+
+
+def test_full_config2_closed_loop_sampled(ctx):
+    """f3 at the bench's size: seq_kernel, one chain per trace over 100,000
+    rounds, decisions and every summary field bit-exact on a sample."""
+    N, T = 4096, 100_000
+    xd = ctx.gen_traces(gen.SEEDS[3], N, T)
+    pols = [magus.make_policy(variant=1)]
+    r = ctx.replay(xd, pols, want_decisions=True)
+    torch.cuda.synchronize()
+    assert ctx.stats()["last_kernel"] == magus.KERNEL_SEQUENTIAL
+    sample = _sample(N, 12, 6)
+    _check_sample(ctx, xd, pols, sample, r)
+    xs = xd[:, torch.as_tensor(sample, device=xd.device)].cpu().numpy()
+    ref = oracle.replay(np.ascontiguousarray(xs), to_oracle_policies(pols), want_dec=True)
+    dec = r.decisions_numpy()
+    for i, n in enumerate(sample):
+        assert np.array_equal(dec[0, :, n], oracle.decision_words(ref.dec[0, i], 8)), n
