@@ -760,8 +760,11 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     const size_t sum_bytes = out_summary ? 0 : align_up(sizeof(magus_summary) * (size_t)(N * C), 256);
     const size_t base_bytes = (out_base || !out_totals) ? 0 : align_up(sizeof(magus_base) * (size_t)N, 256);
     const size_t walk_bytes = walk_scratch_bytes(N, C, T, nseg, ctx->dplat);
-    int32_t max_H = 1;
-    for (int32_t c = 0; c < C; ++c) max_H = std::max(max_H, params[c].history);
+    int32_t max_H = 1, same_W = params[0].window;
+    for (int32_t c = 0; c < C; ++c) {
+      max_H = std::max(max_H, params[c].history);
+      if (params[c].window != same_W) same_W = 0;
+    }
     st = ensure_scratch(ctx, sum_bytes + base_bytes + walk_bytes + 256);
     if (st != MAGUS_OK) return st;
     ctx->work_sig = 0;  // scratch reused: the stream path must re-zero its counters
@@ -774,7 +777,7 @@ static magus_status replay_impl(magus_ctx ctx, const float* traces, int64_t N, i
     const double p_lo = ctx->plat.p_other_w + ctx->plat.p_unc_min_w;
     const double p_span = ctx->plat.p_unc_max_w - ctx->plat.p_unc_min_w;
     int r = launch_walk(ctx->stream, traces, N, T, ld, dev_policies(ctx), C, max_H, ctx->dplat, ctx->plat.bw_max_mbs,
-                        p_lo, p_span, nseg, seg_len, sp, summ, base, out_decisions, out_levels, ctx->opt_walk1 != 0);
+                        p_lo, p_span, nseg, seg_len, sp, summ, base, out_decisions, out_levels, ctx->opt_walk1 != 0, same_W);
     if (r < 0) return cuda_fail(ctx, cudaGetLastError(), "walk kernel launch");
     launched += r;
     ctx->last_grid = ((N + 127) / 128) * nseg * C;

@@ -110,7 +110,11 @@ __device__ __forceinline__ void load_rows(const float* __restrict__ p, int ld32,
 // the paper's order -- Alg. 2 on the H previous events (s >= k <=> RN(s/H)
 // >= t_hi), Alg. 1 (host-inverted thresholds), event logging -- recorded as
 // three bit masks per 32-step word, and composed into the segment's map.
-template <typename HT>
+// WT > 0: every config of the launch has W = WT; a full word loads its 32
+// samples once and takes the Alg. 1 lags x[t-W+1] from a register window
+// (the word's own samples and the previous word's last W-1, each widened to
+// fp64 once), instead of a second row load and conversion per sample.
+template <typename HT, int WT>
 __global__ void __launch_bounds__(kWalkThreads, 5) walk_map_kernel(WalkArgs a, int32_t lmin, int32_t lmax, int32_t nlev) {
   const int64_t n = (int64_t)blockIdx.x * kWalkThreads + threadIdx.x;
   const int32_t s = blockIdx.y, cl = blockIdx.z, c = a.c0 + cl;
@@ -143,6 +147,18 @@ __global__ void __launch_bounds__(kWalkThreads, 5) walk_map_kernel(WalkArgs a, i
   // one round: Alg. 2, Alg. 1, the event log, and the composition with this
   // round's map: hold, +-step (l.18 / l.23-25), or the override to max (l.10)
   // one round: Alg. 2 on the H previous events, Alg. 1, the event log
+  auto round_d = [&](int i, double D) {
+    const bool pi = D > P.d_inc, pd = !pi && D < P.d_dec;
+    inc |= (uint32_t)pi << i;
+    dcr |= (uint32_t)pd << i;
+    if constexpr (!kBits) {
+      const bool hf = __popc((uint32_t)(hist & hmask)) + __popc((uint32_t)((uint64_t)hist >> 32)) >= P.k;
+      hw |= (uint32_t)hf << i;
+      hist = ((hist << 1) | (HT)(pi || pd)) & hmask;
+    }
+  };
+  double pdw[WT > 1 ? WT - 1 : 1];   // WT: x[tw-W+1 .. tw-1], widened (valid when have_pd)
+  bool have_pd = false;
   auto round = [&](int i, float xt, float xl) {
     const double D = (double)xt - (double)xl;
     const bool pi = D > P.d_inc, pd = !pi && D < P.d_dec;
@@ -156,7 +172,25 @@ __global__ void __launch_bounds__(kWalkThreads, 5) walk_map_kernel(WalkArgs a, i
   };
   for (int32_t tw = t0; tw < t1; tw += 32) {
     inc = dcr = hw = 0;
-    if (tw >= P.W && tw + 32 <= t1) {   // a full word of MDFS rounds
+    if (WT > 0 && tw >= P.W && tw + 32 <= t1) {   // a full word, lags from registers
+      const float* px = a.x + (int64_t)tw * a.ld + n;
+      if (!have_pd) {
+#pragma unroll
+        for (int k = 0; k < (WT > 1 ? WT - 1 : 0); ++k) pdw[k] = (double)__ldg(px + (k - (WT - 1)) * ld32);
+        have_pd = true;
+      }
+      float xs[32];
+      load_rows<32>(px, ld32, xs);
+      double xd[32];
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        xd[i] = (double)xs[i];                                   // exact widening, once
+        const double xl = (i >= WT - 1) ? xd[i - (WT > 1 ? WT - 1 : 0)] : pdw[i < WT - 1 ? i : 0];
+        round_d(i, xd[i] - xl);                                 // Alg. 1 l.3 numerator (RN)
+      }
+#pragma unroll
+      for (int k = 0; k < (WT > 1 ? WT - 1 : 0); ++k) pdw[k] = xd[32 - (WT - 1) + k];
+    } else if (tw >= P.W && tw + 32 <= t1) {   // a full word of MDFS rounds
       const float* px = a.x + (int64_t)tw * a.ld + n;
       const float* pl = px - (int64_t)(P.W - 1) * a.ld;
       constexpr int kq = kWalkChunk / 2;  // samples + lags: 16 loads ahead
@@ -171,6 +205,7 @@ __global__ void __launch_bounds__(kWalkThreads, 5) walk_map_kernel(WalkArgs a, i
     } else {                            // warm-up rounds (t < W) / the ragged tail
       for (int32_t t = max(tw, P.W); t < min(tw + 32, t1); ++t)
         round(t - tw, a.x[(int64_t)t * a.ld + n], a.x[(int64_t)(t - P.W + 1) * a.ld + n]);
+      have_pd = false;
     }
     if constexpr (kBits) {
       // rounds of this word that ran Alg. 2: t >= W and t < t1 (inc / dcr
@@ -696,7 +731,7 @@ size_t walk_scratch_bytes(int64_t N, int32_t C, int64_t T, int64_t nseg, const D
 int launch_walk(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld, const DevPolicy* pol_dev,
                 int32_t C, int32_t max_H, const DevPlatform& plat, double bw_max, double p_lo, double p_span,
                 int64_t nseg, int64_t seg_len, void* scratch, magus_summary* out_summary, magus_base* out_base,
-                uint32_t* out_dec, uint8_t* out_levels, bool fused) {
+                uint32_t* out_dec, uint8_t* out_levels, bool fused, int32_t same_W) {
   const int nlev = plat.r_max - plat.r_min + 1;
   const int64_t B = walk_batch(N, C, T), nw = (T + 31) / 32;
   auto al = [](size_t b) { return (b + 255) / 256 * 256; };
@@ -739,7 +774,17 @@ int launch_walk(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld
     lv.bkeep[i] = (plat.burst_on && Bl > plat.burst_mbs) ? 1 : 0;
   }
   int launched = 0;
-  auto mk = max_H > 32 ? walk_map_kernel<uint64_t> : walk_map_kernel<uint32_t>;
+  // one compile-time W for the whole launch when every config shares it
+  auto mk = max_H > 32 ? walk_map_kernel<uint64_t, 0> : walk_map_kernel<uint32_t, 0>;
+  if (max_H <= 32) {
+    switch (same_W) {
+      case 4: mk = walk_map_kernel<uint32_t, 4>; break;
+      case 6: mk = walk_map_kernel<uint32_t, 6>; break;
+      case 10: mk = walk_map_kernel<uint32_t, 10>; break;
+      case 16: mk = walk_map_kernel<uint32_t, 16>; break;
+      default: break;
+    }
+  }
   const size_t cnt_smem = (size_t)nlev * kWalkThreads * sizeof(unsigned int);  // <= 65 KB (127 ratios)
   if (cnt_smem > 48 * 1024) {
     if (cudaFuncSetAttribute(walk_replay_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cnt_smem) !=

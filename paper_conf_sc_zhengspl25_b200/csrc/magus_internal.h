@@ -125,7 +125,8 @@ size_t walk_scratch_bytes(int64_t N, int32_t C, int64_t T, int64_t nseg, const D
 int launch_walk(cudaStream_t s, const float* x, int64_t N, int64_t T, int64_t ld, const DevPolicy* pol_dev,
                 int32_t C, int32_t max_H, const DevPlatform& plat, double bw_max, double p_lo, double p_span,
                 int64_t nseg, int64_t seg_len, void* scratch, magus_summary* out_summary, magus_base* out_base,
-                uint32_t* out_dec, uint8_t* out_levels, bool fused);
+                uint32_t* out_dec, uint8_t* out_levels, bool fused,
+                int32_t same_W /* W of every config, else 0: pass 1's compile-time lag window */);
 
 // Speculatively time-segmented closed loop (kernels_spec.cu): f3 with the
 // jump rule; scratch = spec_scratch_bytes; out_summary required.
