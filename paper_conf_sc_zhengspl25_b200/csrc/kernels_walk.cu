@@ -282,6 +282,7 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
   const DevPolicy P = a.pol[c];
   const int32_t t0 = s * a.seg_len, t1 = min(a.T, t0 + a.seg_len);
   const int step = (P.variant & MAGUS_VARIANT_GRADUAL) ? P.step : (lmax - lmin);
+  const int K = lmax - lmin;
 
   // carry-in dec[t0 - 1]: dec[-1] := r_max (P@23755), then every earlier
   // segment's map
@@ -305,6 +306,23 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
 
   // round i of the word: the step rule from the pass-1 masks (all zero in
   // the warm-up, t < W), and the per-sample flags of interval 32w + i
+  // full words: round i's level offset as a signed byte (+K on the override --
+  // min(l + K, r_max) = r_max -- +-step, 0), byte i % 4 of F[i / 4]; one
+  // sign-extending byte permute per round instead of three bit tests and
+  // selects
+  auto round_f = [&](int i, float xt, uint32_t F) {
+    or_if_gt(big, xt, xthr_cur, 1u << i);     // stretched at its level (sparse)
+    or_if_gt(bmx, xt, xthr_max, 1u << i);     // ... and at r_max (q_base; rarer still)
+    if (BURST) or_if_gt(bst, xt, xburst, 1u << i);
+    int dl;
+    asm("prmt.b32 %0, %1, 0, %2;" : "=r"(dl) : "r"(F), "r"((uint32_t)((i & 3) | ((8 | (i & 3)) * 0x1110))));
+    const int prev = lvl;
+    lvl = min(max(lvl + dl, lmin), lmax);                      // l.10 / l.18-19 / l.23-25
+    s_lv[i][tid] = (uint8_t)lvl;
+    xthr_cur = s_xthr[lvl - lmin];
+    word |= (uint32_t)(lvl == lmin) << i;
+    chg |= (uint32_t)(lvl != prev) << i;
+  };
   auto round = [&](int i, float xt) {
     big |= (uint32_t)(xt > xthr_cur) << i;    // stretched at its level (sparse)
     bmx |= (uint32_t)(xt > xthr_max) << i;    // ... and at r_max (q_base; rarer still)
@@ -332,12 +350,22 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
     const int rem = min(32, t1 - tw);
     const float* px = a.x + (int64_t)tw * a.ld + n;
     if (rem == 32) {
+      // the offset bytes: the masks' bits spread to bytes by a multiply (bit j
+      // of a nibble -> byte j), at most one of up / down / override per round
+      const uint32_t U = inc & ~hw, Dn = dcr & ~hw;
+      auto spread4 = [](uint32_t m) { return (m * 0x00204081u) & 0x01010101u; };
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
         float xs[kWalkChunk];
         load_rows<kWalkChunk>(px + h * kWalkChunk * ld32, ld32, xs);
 #pragma unroll
-        for (int i = 0; i < kWalkChunk; ++i) round(h * kWalkChunk + i, xs[i]);
+        for (int q = 0; q < kWalkChunk / 4; ++q) {
+          const int sh = 4 * (h * (kWalkChunk / 4) + q);
+          const uint32_t F = spread4((U >> sh) & 15u) * (uint32_t)step + spread4((hw >> sh) & 15u) * (uint32_t)K +
+                             spread4((Dn >> sh) & 15u) * (uint32_t)(256 - step);
+#pragma unroll
+          for (int i = 0; i < 4; ++i) round_f(h * kWalkChunk + 4 * q + i, xs[4 * q + i], F);
+        }
       }
     } else {
       for (int i = 0; i < rem; ++i) round(i, __ldg(px + i * ld32));
