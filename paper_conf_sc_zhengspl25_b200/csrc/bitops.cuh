@@ -104,6 +104,12 @@ __device__ __forceinline__ void or_if_lt(uint32_t& w, double a, double b, uint32
   asm("{\n.reg .pred p;\nsetp.lt.f64 p, %1, %2;\n@p or.b32 %0, %0, %3;\n}"
       : "+r"(w) : "d"(a), "d"(b), "r"(bit));
 }
+__device__ __forceinline__ void or_if_eq(uint32_t& w, int a, int b, uint32_t bit) {
+  asm("{\n.reg .pred p;\nsetp.eq.s32 p, %1, %2;\n@p or.b32 %0, %0, %3;\n}" : "+r"(w) : "r"(a), "r"(b), "r"(bit));
+}
+__device__ __forceinline__ void or_if_ne(uint32_t& w, int a, int b, uint32_t bit) {
+  asm("{\n.reg .pred p;\nsetp.ne.s32 p, %1, %2;\n@p or.b32 %0, %0, %3;\n}" : "+r"(w) : "r"(a), "r"(b), "r"(bit));
+}
 __device__ __forceinline__ void or_if_gt(uint32_t& w, float a, float b, uint32_t bit) {
   asm("{\n.reg .pred p;\nsetp.gt.f32 p, %1, %2;\n@p or.b32 %0, %0, %3;\n}"
       : "+r"(w) : "f"(a), "f"(b), "r"(bit));

@@ -266,23 +266,36 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
   __shared__ float s_xthr[kWalkMaxLv];
   __shared__ uint8_t s_bkeep[kWalkMaxLv];
   __shared__ uint8_t s_lv[32][kWalkThreads];  // dec[32w + i] of the current word
+  // level offsets of 4 rounds as signed bytes (byte j: +step up, -step down,
+  // +K the override -- min(l + K, r_max) = r_max --, 0 hold), indexed by the
+  // rounds' (up | override) nibble and, above it, their (down | override) nibble
+  __shared__ uint32_t s_off[256];
   extern __shared__ unsigned int s_cnt[];     // [nlev][kWalkThreads] intervals per level
   const int lmin = plat.r_min, lmax = plat.r_max, nlev = lmax - lmin + 1;
+  const int32_t s = blockIdx.y, cl = blockIdx.z, c = a.c0 + cl;
+  const DevPolicy P = a.pol[c];
+  const int step = (P.variant & MAGUS_VARIANT_GRADUAL) ? P.step : (lmax - lmin);
+  const int K = lmax - lmin;
   for (int i = 0; i < nlev; ++i) s_cnt[i * kWalkThreads + threadIdx.x] = 0u;
   for (int i = threadIdx.x; i < nlev; i += kWalkThreads) {
     s_invB[i] = lv.invB[i];
     s_xthr[i] = lv.xthr[i];
     s_bkeep[i] = lv.bkeep[i];
   }
+  for (int idx = threadIdx.x; idx < 256; idx += kWalkThreads) {
+    uint32_t F = 0;
+    for (int j = 0; j < 4; ++j) {
+      const int code = ((idx >> j) & 1) | (((idx >> (4 + j)) & 1) << 1);
+      const uint32_t b = code == 1 ? (uint32_t)step : (code == 2 ? (uint32_t)(256 - step) : (code == 3 ? (uint32_t)K : 0u));
+      F |= b << (8 * j);
+    }
+    s_off[idx] = F;
+  }
   __syncthreads();
   const int tid = threadIdx.x;
   const int64_t n = (int64_t)blockIdx.x * kWalkThreads + tid;
-  const int32_t s = blockIdx.y, cl = blockIdx.z, c = a.c0 + cl;
   if (n >= a.N) return;
-  const DevPolicy P = a.pol[c];
   const int32_t t0 = s * a.seg_len, t1 = min(a.T, t0 + a.seg_len);
-  const int step = (P.variant & MAGUS_VARIANT_GRADUAL) ? P.step : (lmax - lmin);
-  const int K = lmax - lmin;
 
   // carry-in dec[t0 - 1]: dec[-1] := r_max (P@23755), then every earlier
   // segment's map
@@ -320,8 +333,8 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
     lvl = min(max(lvl + dl, lmin), lmax);                      // l.10 / l.18-19 / l.23-25
     s_lv[i][tid] = (uint8_t)lvl;
     xthr_cur = s_xthr[lvl - lmin];
-    word |= (uint32_t)(lvl == lmin) << i;
-    chg |= (uint32_t)(lvl != prev) << i;
+    or_if_eq(word, lvl, lmin, 1u << i);
+    or_if_ne(chg, lvl, prev, 1u << i);
   };
   auto round = [&](int i, float xt) {
     big |= (uint32_t)(xt > xthr_cur) << i;    // stretched at its level (sparse)
@@ -350,10 +363,10 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
     const int rem = min(32, t1 - tw);
     const float* px = a.x + (int64_t)tw * a.ld + n;
     if (rem == 32) {
-      // the offset bytes: the masks' bits spread to bytes by a multiply (bit j
-      // of a nibble -> byte j), at most one of up / down / override per round
-      const uint32_t U = inc & ~hw, Dn = dcr & ~hw;
-      auto spread4 = [](uint32_t m) { return (m * 0x00204081u) & 0x01010101u; };
+      // the offset bytes of each 4 rounds from the shared table (inc, dcr
+      // exclusive; the override sets both nibbles)
+      const uint32_t clo = inc | hw, chi = dcr | hw;
+      const uint32_t off_s = (uint32_t)__cvta_generic_to_shared(s_off);
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
         float xs[kWalkChunk];
@@ -361,8 +374,9 @@ __global__ void __launch_bounds__(kWalkThreads, 6) walk_replay_kernel(WalkArgs a
 #pragma unroll
         for (int q = 0; q < kWalkChunk / 4; ++q) {
           const int sh = 4 * (h * (kWalkChunk / 4) + q);
-          const uint32_t F = spread4((U >> sh) & 15u) * (uint32_t)step + spread4((hw >> sh) & 15u) * (uint32_t)K +
-                             spread4((Dn >> sh) & 15u) * (uint32_t)(256 - step);
+          const uint32_t idx = ((clo >> sh) & 15u) | (((chi >> sh) & 15u) << 4);
+          uint32_t F;
+          asm("ld.shared.u32 %0, [%1];" : "=r"(F) : "r"(off_s + 4u * idx));
 #pragma unroll
           for (int i = 0; i < 4; ++i) round_f(h * kWalkChunk + 4 * q + i, xs[4 * q + i], F);
         }
