@@ -100,15 +100,18 @@ __device__ __forceinline__ unsigned long long run_sum(uint32_t lv, uint32_t col)
   const uint32_t nx = lv >> 1;
   uint32_t plus = lv & ~nx, minus = ~lv & nx;
   unsigned long long s = 0;
+  // one trip per run: its end and (unless the run starts at 0) the position
+  // before its start -- every minus bit belongs to a run, so popc(minus) <=
+  // popc(plus) and one loop over the runs covers both (half the trips and
+  // loop control of two loops)
   while (plus) {
     const int t = 31 - __clz(plus);
     plus ^= 1u << t;
+    const int tm = 31 - __clz(minus | 1u);               // 0 when no minus bit is left
+    const unsigned long long pm = lds_u64v(col + 256u * (uint32_t)tm);
     s += lds_u64v(col + 256u * (uint32_t)t);
-  }
-  while (minus) {
-    const int t = 31 - __clz(minus);
-    minus ^= 1u << t;
-    s -= lds_u64v(col + 256u * (uint32_t)t);
+    if (minus) s -= pm;
+    minus &= ~(1u << tm);
   }
   return s;
 }
