@@ -375,6 +375,8 @@ family_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
     const uint32_t E = incv | decv;              // uncore_tune_ls.push_back(1)
     if (w >= wt0) {
       const uint32_t outm = (w == w_tail) ? tail_m : ~0u;
+      // the position of the word's last decision: 31, or the trace's last interval
+      const uint32_t lsh = (w == w_tail) ? (uint32_t)((Ti - 1) & 31) : 31u;
       const uint64_t M = lds_u64v(mb_s + (uint32_t)offsetof(MaskBuf, M));
       const uint32_t smin = lds_u32(mb_s + (uint32_t)offsetof(MaskBuf, smin) + 4u * lane);
       const uint32_t xmx = lds_u32(mb_s + (uint32_t)offsetof(MaskBuf, xmx) + 4u * lane);
@@ -409,11 +411,11 @@ family_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
         const uint32_t chm = (Dw ^ Lv) & outm;
         const uint32_t Dout = Dw & outm;
         cnt_a[k] += (uint32_t)__popc(HI & outm) | ((uint32_t)__popc(act & outm) << 16);
-        cnt_b[k] += (uint32_t)__popc(Dout) | ((uint32_t)__popc(Lv & outm) << 16);
+        cnt_b[k] += (uint32_t)__popc(Dout);   // (intervals at min: from the decisions, see the epilogue)
         cnt_c[k] += (uint32_t)__popc(chm);
         dig[k] += (unsigned long long)Dout * M;
         Lvk[k] = Lv;
-        carry = (carry & ~(1u << k)) | ((Dw >> 31) << k);
+        carry = (carry & ~(1u << k)) | (((Dw >> lsh) & 1u) << k);
         if constexpr (DEC) {  // words after the first action (earlier ones are deferred)
           if (valid && ((seen_w >> k) & 1u) && cfg[k] >= 0)
             reinterpret_cast<uint32_t*>(dec_row)[(int64_t)(cfg[k] - c0) * wk.dec_cstride] = Dout;
@@ -514,23 +516,27 @@ family_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
     if (wk.carry && s == nseg - 1)
       st_release(status + s * N, (wk.epoch << 3) | 3u | ((sk ? (carry >> k) & 1u : cin) << 2));
     uint32_t hi = cnt_a[k] & 0xFFFFu, msr = cnt_a[k] >> 16;
-    uint32_t mdec = cnt_b[k] & 0xFFFFu, mint = cnt_b[k] >> 16;
+    uint32_t mdec = cnt_b[k];
     uint32_t ch = cnt_c[k];
     unsigned long long qn = qmin[k], qx = S.qmax, dg = dig[k];
     const unsigned long long pqn = sk ? pqmin[k] : Gb, pqx = sk ? S.pqmax : Gxb;  // no action: the whole segment
     if (cin != hyp) {
-      const uint32_t n_int = sk ? (uint32_t)S.apos + 1u : (uint32_t)(t1 - t0);
       const uint32_t n_dec = sk ? (uint32_t)S.apos : (uint32_t)(t1 - t0);
       if (hyp) {  // assumed min, truly max
-        mint -= n_int; mdec -= n_dec;
+        mdec -= n_dec;
         qn -= pqn; qx += pqx; dg -= S.pdig;
       } else {    // assumed max, truly min
-        mint += n_int; mdec += n_dec;
+        mdec += n_dec;
         qn += pqn; qx -= pqx; dg += S.pdig;
       }
       const uint32_t vak = (va >> k) & 1u;
       if (sk) ch += (uint32_t)((int)(vak != cin) - (int)(vak != hyp));
     }
+    // intervals t0 .. t1-1 run at dec[t0-1] .. dec[t1-2]: the segment's min
+    // decisions, plus the carry-in, minus its last decision (the hold of the
+    // carry when nothing acted) -- the popcount of the interval mask, summed
+    const uint32_t dlast = sk ? (carry >> k) & 1u : cin;
+    const uint32_t mint = mdec + cin - dlast;
     if (want_dec) {  // deferred prefix decision words
       uint32_t* dec_out = wk.dec + (int64_t)c * wk.dec_cstride + n;
       const uint32_t fill = cin ? ~0u : 0u;
