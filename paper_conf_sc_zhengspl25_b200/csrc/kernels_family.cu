@@ -595,10 +595,7 @@ family_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
       if (wk.totals) {  // per-config fleet totals (exact integer sums): one warp = the group's 32 traces
 #pragma unroll
         for (int q = 0; q < kTotAcc; ++q) {
-          unsigned long long v = tv[q];
-#pragma unroll
-          for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xFFFFFFFFu, v, o);
-          tv[q] = v;
+          tv[q] = warp_sum_tot(tv[q], q);
         }
         if (lane == 0) {
           while (ld_acquire(wk.ticket + kTotalsFlagWord) == 0u) __nanosleep(MAGUS_LOOKBACK_SLEEP);

@@ -666,9 +666,7 @@ stream_kernel(const __grid_constant__ CUtensorMap tmap, const __grid_constant__ 
       if (wk.totals) {  // per-config fleet totals (exact integer sums)
 #pragma unroll
         for (int q = 0; q < kTotAcc; ++q) {
-          unsigned long long v = tv[q];
-#pragma unroll
-          for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xFFFFFFFFu, v, o);
+          const unsigned long long v = warp_sum_tot(tv[q], q);
           if (lane == 0) sh_red[warp][q] = v;
         }
         consumer_sync<TR>();

@@ -129,6 +129,18 @@ __device__ __forceinline__ void trace_put(unsigned long long* tr, int i, unsigne
   tr[8ull * cta + i] = v;
 }
 
+// The warp's sum of one per-trace totals field (each lane's value < 2^32):
+// counts (<= T <= 2^24 per trace, so the warp's sum < 2^29) by one
+// redux.sync, the 32-bit halves of the q sums (fields 7..12) by two on
+// 16-bit pieces -- exact, without five rounds of 64-bit shuffles.
+__device__ __forceinline__ unsigned long long warp_sum_tot(unsigned long long v, int q) {
+  const uint32_t v32 = (uint32_t)v;
+  if (q >= 7 && q <= 12)
+    return (unsigned long long)__reduce_add_sync(0xFFFFFFFFu, v32 & 0xFFFFu) +
+           ((unsigned long long)__reduce_add_sync(0xFFFFFFFFu, v32 >> 16) << 16);
+  return (unsigned long long)__reduce_add_sync(0xFFFFFFFFu, v32);
+}
+
 __device__ __forceinline__ uint32_t tail_mask(int64_t p0, int64_t T) {
   return (p0 + 32 <= T) ? ~0u : ((1u << (uint32_t)(T - p0)) - 1u);
 }
