@@ -173,3 +173,20 @@ def test_walk_kernel_rejects_closed_loop():
         ctx.replay_levels(xd, pols)
         torch.cuda.synchronize()
         assert ctx.stats()["last_kernel"] == 3
+
+
+@pytest.mark.parametrize("W", [4, 6, 10, 16])
+@pytest.mark.parametrize("segments", [1, 11, 87])
+def test_walk_kernel_compile_time_window(W, segments):
+    """Every config of the launch shares W in {4, 6, 10, 16}: pass 1 takes
+    the Alg. 1 lags from its register window (segment starts reload it, the
+    warm-up and the ragged tail take the row-load path)."""
+    N, T = 150, 2777
+    x = gen.gen_traces(gen.SEEDS[4], N, T)
+    pols = [magus.make_policy(W=W, variant=2, step=2), magus.make_policy(W=W, H=7, t_hi=0.3, variant=2, step=1),
+            magus.make_policy(W=W, variant=0)]
+    po, pm = _platforms("a100", 12000.0)
+    ref = oracle.replay(x, _opol(pols), po, want_dec=True)
+    with magus.Context(device=0, platform=pm) as ctx:
+        lv, res = _levels(ctx, x, pols, segments)
+    _check(lv, res, ref, po, T, len(pols))
